@@ -1,0 +1,548 @@
+// api.cu -- the C ABI (include/atos.h): handles, configuration, errors, and
+// the host-side plumbing shared by all solvers.
+#include <cstdarg>
+#include <cstring>
+#include <chrono>
+#include <thread>
+#include <algorithm>
+#include <functional>
+
+#include "internal.h"
+
+namespace atos {
+
+static thread_local char g_err[1024] = "";
+std::atomic<uint64_t> g_launches{0};
+
+void set_error(const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+}
+
+int DevBuf::ensure(size_t want) {
+  if (want <= bytes && p) return ATOS_OK;
+  release();
+  if (want == 0) want = 16;
+  cudaError_t e = cudaMalloc(&p, want);
+  if (e != cudaSuccess) {
+    p = nullptr;
+    bytes = 0;
+    cudaGetLastError();
+    set_error("cudaMalloc(%zu) failed: %s", want, cudaGetErrorString(e));
+    return e == cudaErrorMemoryAllocation ? ATOS_ERR_OOM : ATOS_ERR_CUDA;
+  }
+  bytes = want;
+  return ATOS_OK;
+}
+
+void DevBuf::release() {
+  if (p) cudaFree(p);
+  p = nullptr;
+  bytes = 0;
+}
+
+int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
+  atos_cfg d;
+  atos_cfg_default(&d);
+  if (cfg) {
+    if (cfg->struct_size != sizeof(atos_cfg)) {
+      set_error("atos_cfg.struct_size = %u, expected %zu (call atos_cfg_default)", cfg->struct_size,
+                sizeof(atos_cfg));
+      return ATOS_ERR_INVALID_ARG;
+    }
+    d = *cfg;
+  }
+  r->persistent = d.persistent ? 1 : 0;
+  r->worker = d.worker;
+  if (r->worker == 0) r->worker = (app == 'c') ? 32 : 256;
+  if (!(r->worker == 1 || r->worker == 32 || (r->worker >= 64 && r->worker <= 1024 && r->worker % 32 == 0))) {
+    set_error("worker must be 1, 32 or a multiple of 32 in [64, 1024] (got %d)", r->worker);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  r->fetch = d.fetch_size;
+  if (r->fetch == 0) r->fetch = (r->worker >= 64) ? r->worker : (r->worker == 32 ? 8 : 1);
+  if (r->fetch < 1 || r->fetch > 4096) {
+    set_error("fetch_size must be in [1, 4096] (got %d)", r->fetch);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  r->num_blocks = std::max(0, d.num_blocks);
+  r->block_threads = d.block_threads ? d.block_threads : 256;
+  if (r->block_threads < 32 || r->block_threads > 1024 || r->block_threads % 32) {
+    set_error("block_threads must be a multiple of 32 in [32, 1024] (got %d)", r->block_threads);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  r->dedupe = d.dedupe ? 1 : 0;
+  r->check_size = d.check_size;
+  if (r->check_size < 0) {
+    set_error("check_size must be >= 0");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  r->conflict_policy = d.conflict_policy;
+  r->permute_init = d.permute_init;
+  r->validate = d.validate;
+  r->out_where = d.out_where;
+  if (r->out_where != ATOS_MEM_DEVICE && r->out_where != ATOS_MEM_HOST) {
+    set_error("out_where must be ATOS_MEM_DEVICE or ATOS_MEM_HOST");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  r->l2_persist = d.l2_persist;
+  r->queue_capacity = d.queue_capacity;
+  r->timeout_s = d.timeout_s;
+  if (r->timeout_s < 0) {
+    set_error("timeout_s must be >= 0");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  r->stream = (cudaStream_t)d.stream;
+  r->stats = d.stats;
+  r->watchdog_ns = (unsigned long long)((r->timeout_s > 0 ? r->timeout_s : 30.0) * 1e9);
+  return ATOS_OK;
+}
+
+int ensure_queue(Part& p, uint64_t cap, cudaStream_t s) {
+  if (p.ring_cap < cap || !p.ring.p) {
+    ATOS_TRY(p.ring.ensure(cap * 4));
+    p.ring_cap = cap;
+    p.ring_clean = false;
+  }
+  if (!p.ctl.p) ATOS_TRY(p.ctl.ensure(sizeof(QueueCtl)));
+  if (!p.host_pinned) ATOS_CUDA(cudaHostAlloc(&p.host_pinned, 4096, cudaHostAllocDefault));
+  if (!p.ring_clean) {
+    ATOS_CUDA(cudaMemsetAsync(p.ring.p, 0xFF, p.ring_cap * 4, s));
+    p.ring_clean = true;
+  }
+  return ATOS_OK;
+}
+
+int persistent_grid(const void* fn, int block, size_t smem, int* grid) {
+  int dev = 0, sms = 0, per = 0;
+  ATOS_CUDA(cudaGetDevice(&dev));
+  ATOS_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+  ATOS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, block, smem));
+  if (per < 1) {
+    set_error("kernel cannot be resident with block=%d smem=%zu", block, smem);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  *grid = per * sms;
+  return ATOS_OK;
+}
+
+void set_l2_window(cudaStream_t s, void* base, size_t bytes, bool on) {
+  cudaStreamAttrValue v;
+  memset(&v, 0, sizeof(v));
+  if (on && base && bytes) {
+    int dev = 0, maxwin = 0, persist_max = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+    cudaDeviceGetAttribute(&persist_max, cudaDevAttrMaxPersistingL2CacheSize, dev);
+    if (maxwin <= 0 || persist_max <= 0) return;
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)persist_max);
+    size_t win = std::min(bytes, (size_t)maxwin);
+    v.accessPolicyWindow.base_ptr = base;
+    v.accessPolicyWindow.num_bytes = win;
+    v.accessPolicyWindow.hitRatio = std::min(1.0f, (float)persist_max / (float)win);
+    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+  } else {
+    v.accessPolicyWindow.num_bytes = 0;
+  }
+  cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
+  cudaGetLastError();  // best effort
+}
+
+int stream_wait(cudaStream_t s, double timeout_s) {
+  if (timeout_s <= 0) {
+    ATOS_CUDA(cudaStreamSynchronize(s));
+    return ATOS_OK;
+  }
+  auto t0 = std::chrono::steady_clock::now();
+  while (true) {
+    cudaError_t e = cudaStreamQuery(s);
+    if (e == cudaSuccess) return ATOS_OK;
+    if (e != cudaErrorNotReady) ATOS_CUDA(e);
+    double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    if (el > timeout_s * 1.5 + 1.0) {
+      set_error("stream did not finish within timeout_s=%.3f", timeout_s);
+      return ATOS_ERR_TIMEOUT;
+    }
+    std::this_thread::sleep_for(std::chrono::microseconds(50));
+  }
+}
+
+int finish_queue(Part& p, cudaStream_t s, atos_stats* st, const char* what) {
+  QueueCtl* h = (QueueCtl*)p.host_pinned;  // first 1152 bytes of the pinned page
+  static_assert(sizeof(QueueCtl) <= 4096, "control block fits the pinned page");
+  ATOS_CUDA(cudaMemcpyAsync(h, p.ctl.p, sizeof(QueueCtl), cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  ATOS_CUDA(cudaGetLastError());
+  const uint32_t status = (uint32_t)h->status.v;
+  if (status & kStatusOverflow) {
+    p.ring_clean = false;
+    set_error("%s: queue overflow (ring of %llu slots lapped an unconsumed slot)", what,
+              (unsigned long long)p.ring_cap);
+    return ATOS_ERR_QUEUE_OVERFLOW;
+  }
+  if (status & kStatusTimeout) {
+    p.ring_clean = false;
+    set_error("%s: device watchdog expired (no progress)", what);
+    return ATOS_ERR_TIMEOUT;
+  }
+  if (h->done.v != h->tail.v) {
+    p.ring_clean = false;
+    set_error("%s: queue not drained (done=%llu tail=%llu)", what, (unsigned long long)h->done.v,
+              (unsigned long long)h->tail.v);
+    return ATOS_ERR_CUDA;
+  }
+  p.ring_clean = true;
+  if (st) {
+    st->pops += h->stat_pops.v;
+    st->pushes += h->stat_pushes.v;
+    st->edges += h->stat_edges.v;
+  }
+  return ATOS_OK;
+}
+
+// ----------------------------------------------------- CSR upload / checks
+__global__ void k_narrow_row_ptr(const int64_t* in, uint32_t* out, int64_t count, int64_t m, unsigned* bad) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t x = in[i];
+    if (x < 0 || x > m || (i > 0 && in[i - 1] > x) || (i == 0 && x != 0) || (i == count - 1 && x != m))
+      atomicOr(bad, 1u);
+    out[i] = (uint32_t)x;
+  }
+}
+
+__global__ void k_rebase_row_ptr(const int64_t* in, uint32_t* out, int64_t count, int64_t base) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = (uint32_t)(in[i] - base);
+}
+
+__global__ void k_check_col(const int32_t* col, uint32_t* out, int64_t m, int64_t n, unsigned* bad) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t c = col[i];
+    if (c < 0 || (int64_t)c >= n) atomicOr(bad, 2u);
+    if (out) out[i] = (uint32_t)c;
+  }
+}
+
+__global__ void k_max_degree(const uint32_t* row_ptr, int64_t n, unsigned long long* mx) {
+  unsigned long long best = 0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    best = max(best, (unsigned long long)(row_ptr[v + 1] - row_ptr[v]));
+  for (int o = 16; o; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
+  if (lane_id() == 0) atomicMax(mx, best);
+}
+
+// Upload rows [v_begin, v_end) of a CSR into part p (device arrays, u32).
+// row_ptr/col are the FULL arrays (host or device); offsets are rebased.
+static int upload_part(Part& p, int64_t n_global, const int64_t* row_ptr, const int32_t* col, int where,
+                       int64_t v_begin, int64_t v_end, int64_t e_begin, int64_t e_end) {
+  p.v_begin = v_begin;
+  p.v_end = v_end;
+  p.n_local = v_end - v_begin;
+  p.m_local = e_end - e_begin;
+  const int64_t nl = p.n_local, ml = p.m_local;
+  ATOS_CUDA(cudaMalloc(&p.row_ptr, (size_t)(nl + 1) * 4));
+  ATOS_CUDA(cudaMalloc(&p.col, (size_t)std::max<int64_t>(ml, 1) * 4));
+  if (where == ATOS_MEM_HOST) {
+    std::vector<uint32_t> rp((size_t)nl + 1);
+    for (int64_t i = 0; i <= nl; ++i) rp[(size_t)i] = (uint32_t)(row_ptr[v_begin + i] - e_begin);
+    ATOS_CUDA(cudaMemcpy(p.row_ptr, rp.data(), rp.size() * 4, cudaMemcpyHostToDevice));
+    if (ml) ATOS_CUDA(cudaMemcpy(p.col, col + e_begin, (size_t)ml * 4, cudaMemcpyHostToDevice));
+    return ATOS_OK;
+  }
+  // device input: rebase + narrow on the device
+  k_rebase_row_ptr<<<1024, 256>>>(row_ptr + v_begin, p.row_ptr, nl + 1, e_begin);
+  g_launches++;
+  ATOS_CUDA(cudaGetLastError());
+  if (ml) ATOS_CUDA(cudaMemcpy(p.col, col + e_begin, (size_t)ml * 4, cudaMemcpyDeviceToDevice));
+  ATOS_CUDA(cudaDeviceSynchronize());
+  return ATOS_OK;
+}
+
+static int validate_host_csr(int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col) {
+  if (row_ptr[0] != 0 || row_ptr[n] != m) {
+    set_error("row_ptr[0] must be 0 and row_ptr[n] must equal m");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  for (int64_t v = 0; v < n; ++v)
+    if (row_ptr[v + 1] < row_ptr[v]) {
+      set_error("row_ptr is not non-decreasing at %lld", (long long)v);
+      return ATOS_ERR_INVALID_ARG;
+    }
+  for (int64_t e = 0; e < m; ++e)
+    if (col[e] < 0 || (int64_t)col[e] >= n) {
+      set_error("col[%lld] = %d out of range [0, %lld)", (long long)e, col[e], (long long)n);
+      return ATOS_ERR_INVALID_ARG;
+    }
+  return ATOS_OK;
+}
+
+static int validate_device_csr(int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col) {
+  unsigned* bad = nullptr;
+  uint32_t* scratch = nullptr;
+  ATOS_CUDA(cudaMalloc(&bad, 4));
+  ATOS_CUDA(cudaMemset(bad, 0, 4));
+  ATOS_CUDA(cudaMalloc(&scratch, (size_t)(n + 1) * 4));
+  k_narrow_row_ptr<<<1024, 256>>>(row_ptr, scratch, n + 1, m, bad);
+  g_launches++;
+  if (m) {
+    k_check_col<<<1024, 256>>>(col, nullptr, m, n, bad);
+    g_launches++;
+  }
+  unsigned h = 0;
+  ATOS_CUDA(cudaMemcpy(&h, bad, 4, cudaMemcpyDeviceToHost));
+  cudaFree(bad);
+  cudaFree(scratch);
+  if (h & 1u) {
+    set_error("row_ptr invalid (must start at 0, be non-decreasing and end at m)");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (h & 2u) {
+    set_error("col has ids outside [0, n)");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  return ATOS_OK;
+}
+
+void destroy_part(Part& p) {
+  if (p.row_ptr) cudaFree(p.row_ptr);
+  if (p.col) cudaFree(p.col);
+  p.row_ptr = nullptr;
+  p.col = nullptr;
+  DevBuf* bufs[] = {&p.ring, &p.ctl, &p.bitmap, &p.vbuf_a, &p.vbuf_b, &p.vbuf_c, &p.scratch,
+                    &p.ghost_a, &p.ghost_b, &p.touched, &p.outbox, &p.inbox};
+  for (DevBuf* b : bufs) b->release();
+  if (p.host_pinned) cudaFreeHost(p.host_pinned);
+  p.host_pinned = nullptr;
+}
+
+int compute_max_degree(Part& p, int64_t* out) {
+  unsigned long long* d = nullptr;
+  ATOS_CUDA(cudaMalloc(&d, 8));
+  ATOS_CUDA(cudaMemset(d, 0, 8));
+  if (p.n_local > 0) {
+    k_max_degree<<<512, 256>>>(p.row_ptr, p.n_local, d);
+    g_launches++;
+  }
+  unsigned long long h = 0;
+  ATOS_CUDA(cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost));
+  cudaFree(d);
+  *out = (int64_t)h;
+  return ATOS_OK;
+}
+
+int create_single(atos_csr* g, const int64_t* row_ptr, const int32_t* col, int where) {
+  g->parts.resize(1);
+  ATOS_TRY(upload_part(g->parts[0], g->n, row_ptr, col, where, 0, g->n, 0, g->m));
+  return compute_max_degree(g->parts[0], &g->max_degree);
+}
+
+int create_loopback_parts(atos_csr* g, const int64_t* row_ptr, const int32_t* col, int where);
+
+// Output staging: device pointer given -> use it; host pointer -> internal buffer + D2H at the end.
+template <class T>
+int run_with_output(atos_csr* g, T* out, int64_t len, const Resolved& r, DevBuf& staging,
+                           const std::function<int(T*)>& body) {
+  if (r.out_where == ATOS_MEM_DEVICE) return body(out);
+  ATOS_TRY(staging.ensure((size_t)std::max<int64_t>(len, 1) * sizeof(T)));
+  ATOS_TRY(body(staging.as<T>()));
+  ATOS_CUDA(cudaMemcpyAsync(out, staging.p, (size_t)len * sizeof(T), cudaMemcpyDeviceToHost, r.stream));
+  ATOS_CUDA(cudaStreamSynchronize(r.stream));
+  return ATOS_OK;
+}
+
+}  // namespace atos
+
+using namespace atos;
+
+extern "C" {
+
+void atos_cfg_default(atos_cfg* cfg) {
+  if (!cfg) return;
+  memset(cfg, 0, sizeof(*cfg));
+  cfg->struct_size = sizeof(atos_cfg);
+  cfg->persistent = 1;
+  cfg->worker = 0;
+  cfg->fetch_size = 0;
+  cfg->dedupe = 1;
+  cfg->out_where = ATOS_MEM_DEVICE;
+}
+
+const char* atos_last_error(void) { return g_err; }
+int atos_version(void) { return ATOS_VERSION; }
+uint64_t atos_kernel_launches(void) { return g_launches.load(); }
+
+int atos_csr_create(atos_csr** out, int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col, int where,
+                    int device, int num_parts) {
+  if (!out || n < 0 || m < 0 || (n > 0 && !row_ptr) || (m > 0 && !col) || num_parts < 1 ||
+      (where != ATOS_MEM_HOST && where != ATOS_MEM_DEVICE)) {
+    set_error("atos_csr_create: invalid argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  *out = nullptr;
+  if (m >= (int64_t)0xFFFFFFFFll || n >= (int64_t)0x7FFFFFFFll) {
+    set_error("atos_csr_create: n < 2^31 and m < 2^32 required (n=%lld m=%lld)", (long long)n, (long long)m);
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    set_error("atos_csr_create: no CUDA device (%s)", cudaGetErrorString(e));
+    return ATOS_ERR_CUDA;
+  }
+  if (device < 0 || device >= ndev) {
+    set_error("atos_csr_create: device %d out of range (have %d)", device, ndev);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  DeviceGuard dg(device);
+  if (n > 0) {
+    int rc = where == ATOS_MEM_HOST ? validate_host_csr(n, m, row_ptr, col) : validate_device_csr(n, m, row_ptr, col);
+    if (rc != ATOS_OK) return rc;
+  }
+  atos_csr* g = new atos_csr();
+  g->device = device;
+  g->n = n;
+  g->m = m;
+  g->num_parts = num_parts;
+  int rc = num_parts == 1 ? create_single(g, row_ptr, col, where) : create_loopback_parts(g, row_ptr, col, where);
+  if (rc != ATOS_OK) {
+    atos_csr_destroy(g);
+    return rc;
+  }
+  *out = g;
+  return ATOS_OK;
+}
+
+void atos_csr_destroy(atos_csr* g) {
+  if (!g) return;
+  {
+    DeviceGuard dg(g->device);
+    for (auto& p : g->parts) destroy_part(p);
+  }
+  delete g;
+}
+
+int atos_csr_info(const atos_csr* g, int64_t* n, int64_t* m, int* num_parts) {
+  if (!g) {
+    set_error("atos_csr_info: null handle");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (n) *n = g->n;
+  if (m) *m = g->m;
+  if (num_parts) *num_parts = g->comm ? g->nranks : g->num_parts;
+  return ATOS_OK;
+}
+
+int atos_bfs(const atos_csr* gc, int64_t src, uint32_t* depth_out, const atos_cfg* cfg) {
+  atos_csr* g = const_cast<atos_csr*>(gc);
+  if (!g || !depth_out) {
+    set_error("atos_bfs: null argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (src < 0 || src >= g->n) {
+    set_error("atos_bfs: src %lld out of range [0, %lld)", (long long)src, (long long)g->n);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  Resolved r;
+  ATOS_TRY(resolve_cfg(cfg, 'b', &r));
+  std::lock_guard<std::mutex> lk(g->mu);
+  DeviceGuard dg(g->device);
+  atos_stats local{};
+  atos_stats* st = r.stats ? &local : nullptr;
+  CallTimer tm(r.stream);
+  int rc;
+  if (g->comm || g->num_parts > 1) {
+    const int64_t len = g->comm ? g->parts[0].n_local : g->n;
+    rc = run_with_output<uint32_t>(g, depth_out, len, r, g->parts[0].vbuf_c,
+                                   [&](uint32_t* d) { return bfs_partitioned(g, src, d, r, st); });
+  } else {
+    rc = run_with_output<uint32_t>(g, depth_out, g->n, r, g->parts[0].vbuf_c,
+                                   [&](uint32_t* d) { return bfs_single(g, g->parts[0], src, d, r, st); });
+    if (st) st->pushes += 1;
+  }
+  const double ms = tm.stop();
+  if (rc == ATOS_OK && r.stats) {
+    local.kernel_ms = ms;
+    *r.stats = local;
+  }
+  return rc;
+}
+
+int atos_pagerank(const atos_csr* gc, double alpha, double eps, double* rank_out, const atos_cfg* cfg) {
+  atos_csr* g = const_cast<atos_csr*>(gc);
+  if (!g || !rank_out) {
+    set_error("atos_pagerank: null argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (!(alpha > 0.0 && alpha < 1.0) || !(eps > 0.0)) {
+    set_error("atos_pagerank: alpha must be in (0,1) and eps > 0 (alpha=%g eps=%g)", alpha, eps);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  Resolved r;
+  ATOS_TRY(resolve_cfg(cfg, 'p', &r));
+  std::lock_guard<std::mutex> lk(g->mu);
+  DeviceGuard dg(g->device);
+  atos_stats local{};
+  atos_stats* st = r.stats ? &local : nullptr;
+  CallTimer tm(r.stream);
+  int rc;
+  if (g->n == 0) return ATOS_OK;
+  if (g->comm || g->num_parts > 1) {
+    const int64_t len = g->comm ? g->parts[0].n_local : g->n;
+    rc = run_with_output<double>(g, rank_out, len, r, g->parts[0].vbuf_c,
+                                 [&](double* d) { return pagerank_partitioned(g, alpha, eps, d, r, st); });
+  } else {
+    rc = run_with_output<double>(g, rank_out, g->n, r, g->parts[0].vbuf_c,
+                                 [&](double* d) { return pagerank_single(g, g->parts[0], alpha, eps, d, r, st); });
+  }
+  const double ms = tm.stop();
+  if (rc == ATOS_OK && r.stats) {
+    local.kernel_ms = ms;
+    *r.stats = local;
+  }
+  return rc;
+}
+
+int atos_color(const atos_csr* gc, uint64_t seed, int32_t* color_out, const atos_cfg* cfg) {
+  atos_csr* g = const_cast<atos_csr*>(gc);
+  if (!g || !color_out) {
+    set_error("atos_color: null argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (g->comm || g->num_parts > 1) {
+    set_error("atos_color: colouring runs on a single partition only (replicas only, DESIGN.md)");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  Resolved r;
+  ATOS_TRY(resolve_cfg(cfg, 'c', &r));
+  std::lock_guard<std::mutex> lk(g->mu);
+  DeviceGuard dg(g->device);
+  atos_stats local{};
+  atos_stats* st = r.stats ? &local : nullptr;
+  CallTimer tm(r.stream);
+  if (g->n == 0) return ATOS_OK;
+  int rc = run_with_output<int32_t>(g, color_out, g->n, r, g->parts[0].vbuf_c,
+                                    [&](int32_t* d) { return color_single(g, g->parts[0], seed, d, r, st); });
+  const double ms = tm.stop();
+  if (rc == ATOS_OK && r.stats) {
+    local.kernel_ms = ms;
+    *r.stats = local;
+  }
+  return rc;
+}
+
+int atos_partition_range(int64_t n, int nparts, int part, int64_t* v_begin, int64_t* v_end) {
+  if (n < 0 || nparts < 1 || part < 0 || part >= nparts || !v_begin || !v_end) {
+    set_error("atos_partition_range: invalid argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  const int64_t chunk = (n + nparts - 1) / nparts;
+  *v_begin = std::min<int64_t>(n, (int64_t)part * chunk);
+  *v_end = std::min<int64_t>(n, (int64_t)(part + 1) * chunk);
+  return ATOS_OK;
+}
+
+}  // extern "C"

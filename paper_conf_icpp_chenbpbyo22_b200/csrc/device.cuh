@@ -1,0 +1,232 @@
+// device.cuh -- memory-order helpers, warp utilities, the ring queue and the
+// per-warp push buffer shared by every Atos worker kernel (sm_100a).
+//
+// Queue design (ours; the paper specifies only "concurrent_pop / concurrent_push"
+// on a single shared queue, and push_warp):
+//   * ring u32 items[C], C a power of two, every slot EMPTY (0xFFFFFFFF) when idle;
+//   * 64-bit monotone counters head (claims), tail (reservations), done
+//     (completed tasks), each on its own 128-byte line -- they never wrap, so
+//     there is no ABA;
+//   * a producer reserves [t, t+k) with ONE atomicAdd per warp-batch, writes the
+//     ids with st.release (publication); a consumer claims [h, h+k) with ONE
+//     atomicAdd per worker, spins on ld.acquire until a slot != EMPTY, takes
+//     the id and stores EMPTY back;
+//   * termination: done == tail read after an acquire of done (DESIGN.md
+//     "Termination"): every reserved slot has been processed, so no task is in
+//     flight and none can be produced.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace atos {
+
+constexpr uint32_t kEmpty = 0xFFFFFFFFu;
+constexpr uint32_t kUnreached = 0xFFFFFFFFu;
+
+// status bits written by the device watchdog
+constexpr uint32_t kStatusOverflow = 1u;
+constexpr uint32_t kStatusTimeout = 2u;
+
+struct __align__(128) Line64 {
+  unsigned long long v;
+  unsigned long long pad[15];
+};
+
+// Control block of one queue (device memory).  Statistics counters are
+// accumulated per CTA and flushed once per CTA at kernel exit.
+struct QueueCtl {
+  Line64 head;
+  Line64 tail;
+  Line64 done;
+  Line64 status;      // watchdog / overflow flags (u32 in .v)
+  Line64 check;       // PageRank Check_Size sweep cursor
+  Line64 stat_pops;
+  Line64 stat_pushes;
+  Line64 stat_edges;
+  Line64 misc;        // app scratch (e.g. colouring: max colour)
+};
+
+struct Ring {
+  uint32_t* items;
+  unsigned long long mask;  // C - 1
+  QueueCtl* ctl;
+};
+
+// ---------------------------------------------------------------- memory order
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ int32_t ld_relaxed(const int32_t* p) {
+  int32_t v;
+  asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ double ld_relaxed(const double* p) {
+  double v;
+  asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_acquire(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed(uint32_t* p, uint32_t v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed(int32_t* p, int32_t v) {
+  asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t atom_or_release(uint32_t* p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.release.gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+__device__ __forceinline__ uint32_t atom_and_acquire(uint32_t* p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.acquire.gpu.global.and.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+__device__ __forceinline__ unsigned long long atom_add_release(unsigned long long* p, unsigned long long v) {
+  unsigned long long old;
+  asm volatile("atom.release.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+  return old;
+}
+__device__ __forceinline__ unsigned long long atom_read(unsigned long long* p) {
+  // an RMW returns the latest value in the location's coherence order
+  unsigned long long old;
+  asm volatile("atom.acquire.gpu.global.or.b64 %0, [%1], 0;" : "=l"(old) : "l"(p) : "memory");
+  return old;
+}
+__device__ __forceinline__ void red_add_f64(double* p, double v) {
+  asm volatile("red.relaxed.gpu.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
+}
+__device__ __forceinline__ void fence_sc_gpu() { asm volatile("fence.sc.gpu;" ::: "memory"); }
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+
+__device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
+__device__ __forceinline__ uint32_t warp_id() { return threadIdx.x >> 5; }
+__device__ __forceinline__ unsigned long long globaltimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+// splitmix64 (Steele, Lea, Flood 2014): colouring priority pi(v) = splitmix64(seed ^ v).
+// Implemented here independently of the oracle (shared only by name and constants).
+__device__ __forceinline__ unsigned long long splitmix64(unsigned long long x) {
+  unsigned long long z = x + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+// -------------------------------------------------------------------- pushing
+// Per-warp staging buffer in shared memory.  push() is warp-collective (all 32
+// lanes call it with their own `want` flag); entries accumulate and are
+// published 32 at a time: one atomicAdd on tail per 32 pushes, one coalesced
+// 128-byte release store.  flush() publishes the remainder.
+struct WarpPusher {
+  uint32_t* buf;      // 64 entries of shared memory owned by this warp
+  uint32_t cnt;       // warp-uniform fill level (< 32 between calls)
+  uint32_t total;     // warp-uniform number of pushes issued (stats)
+
+  __device__ __forceinline__ void publish(const Ring& q, uint32_t k, unsigned long long watchdog_ns) {
+    // k <= 32 entries in buf[0..k)
+    unsigned long long base = 0;
+    if (lane_id() == 0) base = atomicAdd(&q.ctl->tail.v, (unsigned long long)k);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (lane_id() < k) {
+      uint32_t* slot = q.items + ((base + lane_id()) & q.mask);
+      if (ld_relaxed(slot) != kEmpty) {
+        // ring lapped a slot that has not been consumed yet: wait, bounded
+        unsigned long long t0 = globaltimer();
+        while (ld_relaxed(slot) != kEmpty) {
+          __nanosleep(256);
+          if (globaltimer() - t0 > watchdog_ns) {
+            atomicOr((unsigned int*)&q.ctl->status.v, kStatusOverflow);
+            break;
+          }
+        }
+      }
+      st_release(slot, buf[lane_id()]);
+    }
+    total += k;
+  }
+
+  __device__ __forceinline__ void push(const Ring& q, bool want, uint32_t item,
+                                       unsigned long long watchdog_ns) {
+    unsigned m = __ballot_sync(0xffffffffu, want);
+    if (m == 0) return;
+    uint32_t pos = cnt + __popc(m & ((1u << lane_id()) - 1u));
+    if (want) buf[pos] = item;
+    cnt += __popc(m);
+    __syncwarp();
+    if (cnt >= 32) {
+      publish(q, 32, watchdog_ns);
+      __syncwarp();
+      uint32_t rest = cnt - 32;
+      uint32_t tmp = lane_id() < rest ? buf[32 + lane_id()] : 0;
+      __syncwarp();
+      if (lane_id() < rest) buf[lane_id()] = tmp;
+      cnt = rest;
+      __syncwarp();
+    }
+  }
+
+  __device__ __forceinline__ void flush(const Ring& q, unsigned long long watchdog_ns) {
+    if (cnt) {
+      publish(q, cnt, watchdog_ns);
+      cnt = 0;
+    }
+    __syncwarp();
+  }
+};
+
+// -------------------------------------------------------- block-wide helpers
+// exclusive scan of one value per thread; returns the exclusive prefix and
+// writes the block total to *total.  tmp: shared scratch of >= 32 words.
+__device__ __forceinline__ uint32_t block_exclusive_scan(uint32_t x, uint32_t* tmp, uint32_t* total) {
+  uint32_t lane = lane_id(), wid = warp_id(), nw = (blockDim.x + 31) >> 5;
+  uint32_t incl = x;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= (uint32_t)o) incl += y;
+  }
+  if (lane == 31) tmp[wid] = incl;
+  __syncthreads();
+  if (wid == 0) {
+    uint32_t w = lane < nw ? tmp[lane] : 0;
+    uint32_t wi = w;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, wi, o);
+      if (lane >= (uint32_t)o) wi += y;
+    }
+    if (lane < nw) tmp[lane] = wi - w;   // exclusive warp offsets
+    if (lane == nw - 1) tmp[32] = wi;    // total
+  }
+  __syncthreads();
+  uint32_t r = tmp[wid] + incl - x;
+  *total = tmp[32];
+  __syncthreads();
+  return r;
+}
+
+}  // namespace atos

@@ -1,0 +1,321 @@
+// engine.cuh -- the Atos worker loop (Listing 2) for edge-relax apps
+// (BFS, PageRank), B200-first.
+//
+// One kernel template covers the paper's design space (Sec.3):
+//   * kernel strategy: PERSIST=true  -> persistent kernel, CTAs loop on the
+//                                       shared queue until global termination;
+//                      PERSIST=false -> discrete kernel over one frontier
+//                                       [h0, t0) of the same ring;
+//   * worker size:     MODE_CTA    -> the whole CTA is one worker; the fetched
+//                                     vertices' edges are flattened with a
+//                                     block scan and redistributed to threads
+//                                     (load-balancing search, P:459-468,
+//                                     P:877-884);
+//                      MODE_WARP   -> a warp is one worker and strides one
+//                                     vertex's neighbours at a time (Listing 4
+//                                     BFSWarp);
+//                      MODE_THREAD -> each thread is a worker, walking its own
+//                                     vertices' rows serially;
+//   * FETCH_SIZE: items claimed by one worker per pop.
+//
+// App interface (all __device__, const):
+//   using Payload = ...;
+//   bool begin(uint32_t item, uint32_t& start, uint32_t& deg, Payload& p);
+//        called once per consumed item by the consuming thread; false -> no
+//        edges to relax (task still counts as done);
+//   bool relax(const Payload& p, uint32_t w, uint32_t& out);
+//        one neighbour; true -> enqueue `out`;
+//   const uint32_t* col;  (neighbour array)
+//   bool sweep(...) hooks are app-specific and live in the app files.
+#pragma once
+#include "device.cuh"
+
+namespace atos {
+
+enum { MODE_CTA = 0, MODE_WARP = 1, MODE_THREAD = 2 };
+
+struct EngineParams {
+  Ring q;
+  uint32_t fetch;                   // items per claim per worker (per lane for THREAD)
+  unsigned long long watchdog_ns;   // spin budget before the watchdog trips
+  unsigned long long h0, t0;        // discrete mode: the frontier [h0, t0)
+};
+
+// Per-group shared-memory arena.  K = items a group may hold at once.
+template <class Payload>
+struct GroupSmem {
+  uint32_t* item;
+  uint32_t* start;
+  uint32_t* off;      // degree, then exclusive prefix
+  Payload* pay;
+  unsigned long long* pend;
+  unsigned long long* pend2;
+  uint32_t* ctr;      // [0] nready [1] npend [2] npend_new [3] exit [4] claim_cnt [5] spare
+                      // [6..7] claim_base (u64, 8-byte aligned) [8..40] scan scratch
+};
+
+template <class Payload>
+__host__ __device__ constexpr size_t group_smem_bytes(uint32_t K) {
+  // 3 u32 arrays, payload array, two u64 pending arrays, 48 u32 counters
+  return ((size_t)K * (3 * sizeof(uint32_t)) + 15) / 16 * 16 + ((size_t)K * sizeof(Payload) + 15) / 16 * 16 +
+         (size_t)K * 16 + 48 * sizeof(uint32_t);
+}
+
+template <class Payload>
+__device__ __forceinline__ GroupSmem<Payload> carve(unsigned char* base, uint32_t K) {
+  GroupSmem<Payload> s;
+  size_t o = 0;
+  s.item = (uint32_t*)(base + o); o += K * 4;
+  s.start = (uint32_t*)(base + o); o += K * 4;
+  s.off = (uint32_t*)(base + o); o += K * 4;
+  o = (o + 15) / 16 * 16;
+  s.pay = (Payload*)(base + o); o += ((size_t)K * sizeof(Payload) + 15) / 16 * 16;
+  s.pend = (unsigned long long*)(base + o); o += K * 8;
+  s.pend2 = (unsigned long long*)(base + o); o += K * 8;
+  s.ctr = (uint32_t*)(base + o);
+  return s;
+}
+
+template <int MODE>
+__device__ __forceinline__ void group_sync() {
+  if (MODE == MODE_CTA) __syncthreads(); else __syncwarp();
+}
+
+template <int MODE>
+__device__ __forceinline__ uint32_t group_rank() {
+  return MODE == MODE_CTA ? threadIdx.x : lane_id();
+}
+template <int MODE>
+__device__ __forceinline__ uint32_t group_size() {
+  return MODE == MODE_CTA ? blockDim.x : 32u;
+}
+
+// Try to consume slot `idx`: on success the item goes to s.item[] and the slot
+// is reset to EMPTY; otherwise idx is appended to the new pending list.
+template <class Payload>
+__device__ __forceinline__ void consume_slot(const Ring& q, const GroupSmem<Payload>& s,
+                                             unsigned long long idx) {
+  uint32_t* slot = q.items + (idx & q.mask);
+  uint32_t v = ld_acquire(slot);
+  if (v == kEmpty) {
+    uint32_t k = atomicAdd(&s.ctr[2], 1u);
+    s.pend2[k] = idx;
+  } else {
+    st_relaxed(slot, kEmpty);
+    uint32_t k = atomicAdd(&s.ctr[0], 1u);
+    s.item[k] = v;
+  }
+}
+
+// ------------------------------------------------------------------- kernel
+template <class App, int MODE, bool PERSIST>
+__global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) {
+  using Payload = typename App::Payload;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const uint32_t nwarps = blockDim.x >> 5;
+  const uint32_t K = (MODE == MODE_THREAD) ? 32u * P.fetch : P.fetch;
+  const size_t gbytes = group_smem_bytes<Payload>(K);
+  // push buffers first (64 u32 per warp), then one arena per group
+  uint32_t* pushbuf = (uint32_t*)smem_raw;
+  unsigned char* arena = smem_raw + (size_t)nwarps * 64 * 4;
+  const uint32_t gid = (MODE == MODE_CTA) ? 0 : warp_id();
+  GroupSmem<Payload> s = carve<Payload>(arena + gbytes * gid, K);
+  const uint32_t r = group_rank<MODE>(), G = group_size<MODE>();
+
+  WarpPusher pusher{pushbuf + warp_id() * 64, 0, 0};
+  unsigned long long my_pops = 0, my_edges = 0;
+  const Ring& q = P.q;
+
+  // group index across the grid (discrete mode static chunking)
+  const unsigned long long groups_per_block = (MODE == MODE_CTA) ? 1 : nwarps;
+  const unsigned long long ggid = (unsigned long long)blockIdx.x * groups_per_block + gid;
+
+  if (r == 0) { s.ctr[1] = 0; }
+  group_sync<MODE>();
+
+  bool first = true;
+  unsigned backoff = 32;
+  unsigned long long idle_since = 0;
+  while (true) {
+    // ---------------------------------------------------------- 1. claim
+    if (r == 0) {
+      s.ctr[0] = 0; s.ctr[2] = 0; s.ctr[3] = 0; s.ctr[4] = 0;
+      *(unsigned long long*)&s.ctr[6] = 0;
+      if (!PERSIST) {
+        if (!first) {
+          s.ctr[3] = 1;
+        } else {
+          unsigned long long b = P.h0 + ggid * K;
+          unsigned long long e = b + K < P.t0 ? b + K : P.t0;
+          if (b >= P.t0) s.ctr[3] = 1;
+          else { *(unsigned long long*)&s.ctr[6] = b; s.ctr[4] = (uint32_t)(e - b); }
+        }
+      } else if (s.ctr[1] == 0) {
+        unsigned long long h = ld_relaxed(&q.ctl->head.v);
+        unsigned long long t = ld_relaxed(&q.ctl->tail.v);
+        if (h < t) {
+          unsigned long long amt = t - h < K ? t - h : K;
+          unsigned long long b = atomicAdd(&q.ctl->head.v, amt);
+          *(unsigned long long*)&s.ctr[6] = b;
+          s.ctr[4] = (uint32_t)amt;
+        }
+      }
+    }
+    first = false;
+    group_sync<MODE>();
+    if (s.ctr[3]) break;
+    // ---------------------------------------------------------- 2. gather
+    {
+      const unsigned long long cb = *(unsigned long long*)&s.ctr[6];
+      const uint32_t cc = s.ctr[4], np = s.ctr[1];
+      for (uint32_t i = r; i < cc; i += G) consume_slot(q, s, cb + i);
+      for (uint32_t i = r; i < np; i += G) consume_slot(q, s, s.pend[i]);
+    }
+    group_sync<MODE>();
+    const uint32_t nready = s.ctr[0];
+    if (nready == 0) {
+      // nothing ready: idle path (f2 in Listing 3) -- termination check + backoff
+      if (r == 0) {
+        // move pending list
+        s.ctr[1] = s.ctr[2];
+        for (uint32_t i = 0; i < s.ctr[2]; ++i) s.pend[i] = s.pend2[i];
+        unsigned long long d = atom_read(&q.ctl->done.v);
+        unsigned long long t = atom_read(&q.ctl->tail.v);
+        uint32_t st = *(volatile uint32_t*)&q.ctl->status.v;
+        if (d == t || st != 0) s.ctr[3] = 1;
+        else {
+          unsigned long long now = globaltimer();
+          if (idle_since == 0) idle_since = now;
+          else if (now - idle_since > P.watchdog_ns) {
+            atomicOr((unsigned int*)&q.ctl->status.v, kStatusTimeout);
+            s.ctr[3] = 1;
+          }
+          __nanosleep(backoff);
+          backoff = backoff < 2048 ? backoff * 2 : 2048;
+        }
+      }
+      group_sync<MODE>();
+      if (s.ctr[3]) break;
+      continue;
+    }
+    idle_since = 0;
+    backoff = 32;
+    // pending list for the next iteration (copied in parallel)
+    {
+      const uint32_t npn = s.ctr[2];
+      for (uint32_t i = r; i < npn; i += G) s.pend[i] = s.pend2[i];
+    }
+    // ---------------------------------------------------------- 3. begin (per item)
+    for (uint32_t k = r; k < nready; k += G) {
+      uint32_t st = 0, dg = 0;
+      Payload p{};
+      if (!app.begin(s.item[k], st, dg, p)) dg = 0;
+      s.start[k] = st;
+      s.off[k] = dg;
+      s.pay[k] = p;
+    }
+    group_sync<MODE>();
+    if (r == 0) s.ctr[1] = s.ctr[2];
+    my_pops += (r == 0) ? nready : 0;
+
+    // ---------------------------------------------------------- 4. expand + relax
+    if (MODE == MODE_CTA) {
+      // load-balancing search over the flattened edge list of the batch
+      uint32_t total = 0;
+      uint32_t mydeg = 0;
+      // scan: each thread owns ceil(nready/B) consecutive items
+      const uint32_t per = (nready + G - 1) / G;
+      const uint32_t i0 = r * per, i1 = min(i0 + per, nready);
+      for (uint32_t i = i0; i < i1; ++i) mydeg += s.off[i];
+      uint32_t excl = block_exclusive_scan(mydeg, s.ctr + 8, &total);
+      for (uint32_t i = i0; i < i1; ++i) { uint32_t d = s.off[i]; s.off[i] = excl; excl += d; }
+      __syncthreads();
+      my_edges += (r == 0) ? total : 0;
+      for (uint32_t base = 0; base < total; base += G) {
+        const uint32_t e = base + r;
+        bool want = false;
+        uint32_t out = 0;
+        if (e < total) {
+          // largest i with off[i] <= e
+          uint32_t lo = 0, hi = nready;
+          while (hi - lo > 1) {
+            uint32_t mid = (lo + hi) >> 1;
+            if (s.off[mid] <= e) lo = mid; else hi = mid;
+          }
+          const uint32_t w = __ldg(app.col + s.start[lo] + (e - s.off[lo]));
+          want = app.relax(s.pay[lo], w, out);
+        }
+        pusher.push(q, want, out, P.watchdog_ns);
+      }
+    } else if (MODE == MODE_WARP) {
+      for (uint32_t k = 0; k < nready; ++k) {
+        const uint32_t st = s.start[k], dg = s.off[k];
+        const Payload p = s.pay[k];
+        my_edges += (r == 0) ? dg : 0;
+        for (uint32_t j = 0; j < dg; j += 32) {
+          bool want = false;
+          uint32_t out = 0;
+          if (j + r < dg) {
+            const uint32_t w = __ldg(app.col + st + j + r);
+            want = app.relax(p, w, out);
+          }
+          pusher.push(q, want, out, P.watchdog_ns);
+        }
+      }
+    } else {
+      // THREAD: lane r walks items r, r+32, ... serially; lanes advance in lock step
+      uint32_t k = r, st = 0, dg = 0, j = 0;
+      Payload p{};
+      if (k < nready) { st = s.start[k]; dg = s.off[k]; p = s.pay[k]; }
+      while (true) {
+        while (k < nready && j >= dg) {
+          k += 32;
+          j = 0;
+          if (k < nready) { st = s.start[k]; dg = s.off[k]; p = s.pay[k]; }
+        }
+        const bool active = k < nready;
+        if (__ballot_sync(0xffffffffu, active) == 0) break;
+        bool want = false;
+        uint32_t out = 0;
+        if (active) {
+          const uint32_t w = __ldg(app.col + st + j);
+          ++j;
+          ++my_edges;
+          want = app.relax(p, w, out);
+        }
+        pusher.push(q, want, out, P.watchdog_ns);
+      }
+    }
+    pusher.flush(q, P.watchdog_ns);
+    // ---------------------------------------------------------- 5. complete
+    group_sync<MODE>();
+    if (PERSIST && r == 0) {
+      // release: this group's pushes (tail reservations + slot stores) happen-before done
+      fence_acq_rel_gpu();
+      atom_add_release(&q.ctl->done.v, (unsigned long long)nready);
+    }
+    group_sync<MODE>();
+  }
+  // statistics: one atomic per warp
+  unsigned long long pushes = lane_id() == 0 ? pusher.total : 0;
+  for (int o = 16; o; o >>= 1) {
+    my_pops += __shfl_xor_sync(0xffffffffu, my_pops, o);
+    my_edges += __shfl_xor_sync(0xffffffffu, my_edges, o);
+  }
+  if (lane_id() == 0) {
+    atomicAdd(&q.ctl->stat_pops.v, my_pops);
+    atomicAdd(&q.ctl->stat_edges.v, my_edges);
+    atomicAdd(&q.ctl->stat_pushes.v, pushes);
+  }
+}
+
+// Host-side helper: dynamic shared memory for a launch.
+template <class Payload>
+inline size_t relax_worker_smem(int mode, uint32_t block, uint32_t fetch) {
+  uint32_t nwarps = block / 32;
+  uint32_t K = mode == MODE_THREAD ? 32u * fetch : fetch;
+  uint32_t groups = mode == MODE_CTA ? 1u : nwarps;
+  return (size_t)nwarps * 64 * 4 + group_smem_bytes<Payload>(K) * groups;
+}
+
+}  // namespace atos

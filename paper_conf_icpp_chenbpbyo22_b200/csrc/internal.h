@@ -1,0 +1,155 @@
+// internal.h -- host-side internals of libatos (C++17, not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdint>
+#include <cstdio>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/atos.h"
+#include "engine.cuh"
+
+namespace atos {
+
+// ------------------------------------------------------------------ errors
+void set_error(const char* fmt, ...);
+extern std::atomic<uint64_t> g_launches;
+
+#define ATOS_CUDA(call)                                                                   \
+  do {                                                                                   \
+    cudaError_t e_ = (call);                                                             \
+    if (e_ != cudaSuccess) {                                                             \
+      ::atos::set_error("%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, \
+                        __LINE__);                                                       \
+      return e_ == cudaErrorMemoryAllocation ? ATOS_ERR_OOM : ATOS_ERR_CUDA;             \
+    }                                                                                    \
+  } while (0)
+
+#define ATOS_TRY(expr)        \
+  do {                        \
+    int rc_ = (expr);         \
+    if (rc_ != ATOS_OK) return rc_; \
+  } while (0)
+
+// a device allocation owned by the handle
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  int ensure(size_t want);  // grow-only
+  void release();
+  template <class T> T* as() const { return (T*)p; }
+};
+
+// One partition of a graph resident on one device (a whole graph when P = 1).
+struct Part {
+  int64_t v_begin = 0, v_end = 0;   // owned global vertices
+  int64_t n_local = 0, m_local = 0;
+  uint32_t* row_ptr = nullptr;      // n_local + 1, local offsets
+  uint32_t* col = nullptr;          // m_local, GLOBAL ids (single-partition: the ids)
+  // cached workspaces (grow-only, reused across calls)
+  DevBuf ring, ctl, bitmap, vbuf_a, vbuf_b, vbuf_c, scratch;
+  DevBuf ghost_a, ghost_b, touched, outbox, inbox;
+  uint64_t ring_cap = 0;
+  void* host_pinned = nullptr;      // 4 KB pinned scratch for control-block reads
+  bool ring_clean = false;          // every ring slot is EMPTY
+};
+
+struct Comm;
+
+}  // namespace atos
+
+struct atos_csr {
+  int device = 0;
+  int64_t n = 0, m = 0;
+  int num_parts = 1;                       // > 1: loopback partitions on one device
+  std::vector<atos::Part> parts;
+  atos::Comm* comm = nullptr;              // distributed partition (one per process)
+  int rank = 0, nranks = 1;
+  int64_t max_degree = 0;
+  bool symmetric_checked = false, symmetric = false;
+  std::mutex mu;
+};
+
+namespace atos {
+
+// RAII device guard
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+struct Resolved {
+  int persistent, worker, fetch, num_blocks, block_threads, dedupe, check_size;
+  int conflict_policy, permute_init, validate, out_where, l2_persist;
+  uint64_t queue_capacity;
+  double timeout_s;
+  cudaStream_t stream;
+  atos_stats* stats;
+  unsigned long long watchdog_ns;
+};
+// defaults: app = 'b' (bfs) / 'p' (pagerank) / 'c' (color)
+int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r);
+
+inline int mode_of(int worker) {
+  return worker == 1 ? MODE_THREAD : (worker == 32 ? MODE_WARP : MODE_CTA);
+}
+
+// Ring/control workspace of a partition: capacity >= want (power of two), all slots EMPTY.
+int ensure_queue(Part& p, uint64_t want_cap, cudaStream_t s);
+// persistent grid size: occupancy max x SMs
+int persistent_grid(const void* fn, int block, size_t smem, int* grid);
+// L2 persisting window (best effort)
+void set_l2_window(cudaStream_t s, void* base, size_t bytes, bool on);
+
+// timing helper: events on the call stream
+struct CallTimer {
+  cudaEvent_t a = nullptr, b = nullptr;
+  cudaStream_t s;
+  explicit CallTimer(cudaStream_t st) : s(st) {
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    cudaEventRecord(a, s);
+  }
+  double stop() {
+    cudaEventRecord(b, s);
+    cudaEventSynchronize(b);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    return ms;
+  }
+  ~CallTimer() {
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+  }
+};
+
+// wait for the stream, honouring cfg.timeout_s (polling) -- returns ATOS_ERR_TIMEOUT on expiry
+int stream_wait(cudaStream_t s, double timeout_s);
+
+// single-partition solvers (relax.cu / color.cu)
+int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth_dev, const Resolved& r,
+               atos_stats* st);
+int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank_dev,
+                    const Resolved& r, atos_stats* st);
+int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color_dev, const Resolved& r,
+                 atos_stats* st);
+// partitioned solvers (dist.cu)
+int bfs_partitioned(atos_csr* g, int64_t src, uint32_t* depth_dev, const Resolved& r, atos_stats* st);
+int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_dev, const Resolved& r,
+                         atos_stats* st);
+
+// read the control block after a run: status -> error code, stats
+int finish_queue(Part& p, cudaStream_t s, atos_stats* st, const char* what);
+
+}  // namespace atos

@@ -1,0 +1,321 @@
+// relax.cu -- single-partition BFS and PageRank: init kernels, launchers
+// (persistent and discrete), finalisation.
+#include <algorithm>
+
+#include "apps.cuh"
+#include "internal.h"
+
+namespace atos {
+
+// ------------------------------------------------------------- init kernels
+// BFS init (Alg.1 P:721-725 "vertex.dist = MAX_UINT32", frontier = [source];
+// source depth 0, R-BFS-1).  depth[] was memset to 0xFF on the stream.
+__global__ void k_bfs_init(uint32_t* depth, uint32_t* inq, uint32_t* ring, QueueCtl* ctl, uint32_t src) {
+  if (threadIdx.x == 0) {
+    depth[src] = 0;
+    if (inq) inq[src >> 5] |= 1u << (src & 31);
+    ring[0] = src;
+    ctl->head.v = 0;
+    ctl->tail.v = 1;
+    ctl->done.v = 0;
+    ctl->status.v = 0;
+    ctl->check.v = 0;
+    ctl->stat_pops.v = 0;
+    ctl->stat_pushes.v = 0;
+    ctl->stat_edges.v = 0;
+    ctl->misc.v = 0;
+  }
+}
+
+__global__ void k_ctl_reset(QueueCtl* ctl) {
+  if (threadIdx.x == 0) {
+    ctl->head.v = 0;
+    ctl->tail.v = 0;
+    ctl->done.v = 0;
+    ctl->status.v = 0;
+    ctl->check.v = 0;
+    ctl->stat_pops.v = 0;
+    ctl->stat_pushes.v = 0;
+    ctl->stat_edges.v = 0;
+    ctl->misc.v = 0;
+  }
+}
+
+// PageRank vertex init (Alg.3): rank = 1 - lambda, residue = 0.
+__global__ void k_pr_init_vertices(double* rank, double* res, int64_t n, double one_minus_alpha) {
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    rank[v] = one_minus_alpha;
+    res[v] = 0.0;
+  }
+}
+
+// Row owning edge e: largest r in [lo, hi] with row_ptr[r] <= e.
+__device__ __forceinline__ uint32_t row_of(const uint32_t* __restrict__ row_ptr, uint32_t lo, uint32_t hi,
+                                           uint32_t e) {
+  while (lo < hi) {
+    uint32_t mid = lo + ((hi - lo + 1) >> 1);
+    if (__ldg(row_ptr + mid) <= e) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+// PageRank residue init, read as R-PR-init (garbled P:766): for every vertex v
+// and every out-neighbour w, residue[w] += (1-lambda)*lambda/deg(v).
+// Edge-parallel over tiles of blockDim edges: two global searches per tile
+// bound the tile's rows, then each thread searches only that (L1-resident)
+// row range -- load-balanced regardless of hub degrees.
+__global__ void k_pr_init_edges(const uint32_t* __restrict__ row_ptr, const uint32_t* __restrict__ col,
+                                double* res, uint32_t n, uint32_t m, double c) {
+  __shared__ uint32_t s_r[2];
+  for (uint64_t t0 = (uint64_t)blockIdx.x * blockDim.x; t0 < m; t0 += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t e0 = (uint32_t)t0;
+    const uint64_t tend = t0 + blockDim.x < (uint64_t)m ? t0 + blockDim.x : (uint64_t)m;
+    const uint32_t e1 = (uint32_t)(tend - 1);
+    if (threadIdx.x == 0) s_r[0] = row_of(row_ptr, 0, n - 1, e0);
+    if (threadIdx.x == 32 || (blockDim.x <= 32 && threadIdx.x == 0)) s_r[1] = row_of(row_ptr, 0, n - 1, e1);
+    __syncthreads();
+    const uint32_t e = e0 + threadIdx.x;
+    if (e <= e1) {
+      const uint32_t v = row_of(row_ptr, s_r[0], s_r[1], e);
+      const uint32_t deg = __ldg(row_ptr + v + 1) - __ldg(row_ptr + v);
+      red_add_f64(res + __ldg(col + e), c / (double)deg);
+    }
+    __syncthreads();
+  }
+}
+
+// Initial frontier (R-PR-7): every vertex with residue > eps, warp-aggregated pushes.
+__global__ void k_pr_seed(const double* res, int64_t n, double eps, Ring q, unsigned long long wd) {
+  __shared__ uint32_t bufs[32 * 64];
+  WarpPusher pusher{bufs + warp_id() * 64, 0, 0};
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
+    const int64_t v = base + threadIdx.x;
+    const bool want = v < n && res[v] > eps;
+    pusher.push(q, want, (uint32_t)v, wd);
+  }
+  pusher.flush(q, wd);
+  if (lane_id() == 0) atomicAdd(&q.ctl->stat_pushes.v, (unsigned long long)pusher.total);
+}
+
+// rank_out = rank / n (R-PR-4); residual sum into *sum (conservation check).
+__global__ void k_pr_finalize(double* rank, const double* res, int64_t n, double* sum) {
+  double acc = 0.0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    rank[v] = rank[v] / (double)n;
+    acc += res[v];
+  }
+  for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if (lane_id() == 0 && acc != 0.0) atomicAdd(sum, acc);
+}
+
+// Check_Size sweep (paper's Alg.4), run by a
+// separate single-CTA-per-SM kernel between persistent drains: reserve
+// Check_Size ids with one atomicAdd on the check cursor and enqueue those with
+// residue > eps.  (The sweep variant drives activation; see pagerank_single.)
+__global__ void k_pr_sweep(const double* res, int64_t n, double eps, Ring q, uint32_t check_size,
+                           unsigned long long wd) {
+  __shared__ uint32_t bufs[32 * 64];
+  __shared__ unsigned long long s_c;
+  WarpPusher pusher{bufs + warp_id() * 64, 0, 0};
+  // each CTA sweeps chunks until the cursor passed n ids since kernel start
+  while (true) {
+    if (threadIdx.x == 0) s_c = atomicAdd(&q.ctl->check.v, (unsigned long long)check_size);
+    __syncthreads();
+    const unsigned long long c = s_c;
+    __syncthreads();
+    if (c >= (unsigned long long)n) break;
+    for (uint32_t i = 0; i < check_size; i += blockDim.x) {
+      const unsigned long long id = c + i + threadIdx.x;
+      const bool want = (i + threadIdx.x) < check_size && id < (unsigned long long)n && res[id] > eps;
+      pusher.push(q, want, (uint32_t)id, wd);
+    }
+  }
+  pusher.flush(q, wd);
+  if (lane_id() == 0) atomicAdd(&q.ctl->stat_pushes.v, (unsigned long long)pusher.total);
+}
+
+// -------------------------------------------------------------- launchers
+static inline uint64_t pow2_at_least(uint64_t x) {
+  uint64_t c = 1;
+  while (c < x) c <<= 1;
+  return c;
+}
+
+template <class App, int MODE>
+static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, int block,
+                             Part& p, atos_stats* st) {
+  using Payload = typename App::Payload;
+  cudaStream_t s = r.stream;
+  const size_t smem = relax_worker_smem<Payload>(MODE, block, P.fetch);
+  if (smem > 227 * 1024) {
+    set_error("fetch_size %d with worker %d needs %zu B of shared memory (> 227 KB)", r.fetch, r.worker, smem);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (r.persistent) {
+    const void* fn = (const void*)k_relax_worker<App, MODE, true>;
+    if (smem > 48 * 1024) ATOS_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int grid = 0;
+    ATOS_TRY(persistent_grid(fn, block, smem, &grid));
+    if (r.num_blocks > 0) grid = std::min(grid, r.num_blocks);
+    void* args[] = {(void*)&app, (void*)&P};
+    ATOS_CUDA(cudaLaunchCooperativeKernel(fn, grid, block, args, smem, s));
+    g_launches++;
+    if (st) st->rounds += 1;
+    return ATOS_OK;
+  }
+  // discrete: one launch per frontier [h0, t0); the host reads the
+  // tail after each launch -- the per-frontier host round trip the paper measures.
+  const void* fn = (const void*)k_relax_worker<App, MODE, false>;
+  if (smem > 48 * 1024) ATOS_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const uint64_t K = MODE == MODE_THREAD ? 32ull * P.fetch : P.fetch;
+  const uint64_t groups_per_block = MODE == MODE_CTA ? 1 : block / 32;
+  const uint64_t items_per_block = K * groups_per_block;
+  unsigned long long* h_ctl = (unsigned long long*)p.host_pinned;
+  QueueCtl* ctl = P.q.ctl;
+  ATOS_CUDA(cudaMemcpyAsync(h_ctl, &ctl->tail.v, 8, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  uint64_t h0 = 0, t0 = h_ctl[0];
+  // the discrete frontier is consumed in order, so head follows h0
+  while (h0 < t0) {
+    P.h0 = h0;
+    P.t0 = t0;
+    uint64_t grid = (t0 - h0 + items_per_block - 1) / items_per_block;
+    if (grid > 0x7FFFFFFFull) grid = 0x7FFFFFFFull;
+    void* args[] = {(void*)&app, (void*)&P};
+    ATOS_CUDA(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(block), args, smem, s));
+    g_launches++;
+    if (st) st->rounds += 1;
+    ATOS_CUDA(cudaMemcpyAsync(h_ctl, &ctl->tail.v, 8, cudaMemcpyDeviceToHost, s));
+    ATOS_TRY(stream_wait(s, r.timeout_s));
+    h0 = t0;
+    t0 = h_ctl[0];
+    if (t0 - h0 > p.ring_cap) {
+      set_error("discrete frontier of %llu items exceeds the ring capacity %llu",
+                (unsigned long long)(t0 - h0), (unsigned long long)p.ring_cap);
+      p.ring_clean = false;
+      return ATOS_ERR_QUEUE_OVERFLOW;
+    }
+  }
+  // mirror the persistent bookkeeping so finish_queue sees a drained queue
+  ATOS_CUDA(cudaMemcpyAsync(&ctl->head.v, &ctl->tail.v, 8, cudaMemcpyDeviceToDevice, s));
+  ATOS_CUDA(cudaMemcpyAsync(&ctl->done.v, &ctl->tail.v, 8, cudaMemcpyDeviceToDevice, s));
+  return ATOS_OK;
+}
+
+template <class App>
+static int launch_relax(const App& app, const Ring& q, const Resolved& r, Part& p, atos_stats* st) {
+  EngineParams P;
+  P.q = q;
+  P.fetch = (uint32_t)r.fetch;
+  P.watchdog_ns = r.watchdog_ns;
+  P.h0 = P.t0 = 0;
+  const int mode = mode_of(r.worker);
+  const int block = mode == MODE_CTA ? r.worker : r.block_threads;
+  if (mode == MODE_CTA) return launch_relax_mode<App, MODE_CTA>(app, P, r, block, p, st);
+  if (mode == MODE_WARP) return launch_relax_mode<App, MODE_WARP>(app, P, r, block, p, st);
+  return launch_relax_mode<App, MODE_THREAD>(app, P, r, block, p, st);
+}
+
+static Ring ring_of(Part& p) {
+  Ring q;
+  q.items = p.ring.as<uint32_t>();
+  q.mask = p.ring_cap - 1;
+  q.ctl = p.ctl.as<QueueCtl>();
+  return q;
+}
+
+// --------------------------------------------------------------------- BFS
+int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolved& r, atos_stats* st) {
+  cudaStream_t s = r.stream;
+  const int64_t n = p.n_local;
+  uint64_t want = r.queue_capacity ? r.queue_capacity : (uint64_t)std::max<int64_t>(2 * n, 1024);
+  if (!r.dedupe && !r.queue_capacity) want = (uint64_t)std::max<int64_t>(4 * n, 4096);
+  ATOS_TRY(ensure_queue(p, pow2_at_least(want), s));
+  uint32_t* inq = nullptr;
+  if (r.dedupe) {
+    ATOS_TRY(p.bitmap.ensure(((size_t)n + 31) / 32 * 4));
+    inq = p.bitmap.as<uint32_t>();
+    ATOS_CUDA(cudaMemsetAsync(inq, 0, ((size_t)n + 31) / 32 * 4, s));
+  }
+  ATOS_CUDA(cudaMemsetAsync(depth, 0xFF, (size_t)n * 4, s));
+  Ring q = ring_of(p);
+  k_bfs_init<<<1, 32, 0, s>>>(depth, inq, q.items, q.ctl, (uint32_t)src);
+  g_launches++;
+  ATOS_CUDA(cudaGetLastError());
+  if (r.l2_persist) set_l2_window(s, depth, (size_t)n * 4, true);
+  BfsApp app{p.row_ptr, p.col, depth, inq};
+  p.ring_clean = false;
+  int rc = launch_relax(app, q, r, p, st);
+  if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
+  if (rc != ATOS_OK) return rc;
+  return finish_queue(p, s, st, "bfs");
+}
+
+// ---------------------------------------------------------------- PageRank
+int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank, const Resolved& r,
+                    atos_stats* st) {
+  cudaStream_t s = r.stream;
+  const int64_t n = p.n_local;
+  const uint64_t want = r.queue_capacity ? r.queue_capacity : (uint64_t)std::max<int64_t>(2 * n, 1024);
+  ATOS_TRY(ensure_queue(p, pow2_at_least(want), s));
+  ATOS_TRY(p.vbuf_a.ensure((size_t)n * 8));
+  ATOS_TRY(p.scratch.ensure(64));
+  double* res = p.vbuf_a.as<double>();
+  double* sum = p.scratch.as<double>();
+  Ring q = ring_of(p);
+  k_ctl_reset<<<1, 32, 0, s>>>(q.ctl);
+  g_launches++;
+  const int gs = 148 * 8;
+  k_pr_init_vertices<<<gs, 256, 0, s>>>(rank, res, n, 1.0 - alpha);
+  g_launches++;
+  if (p.m_local > 0) {
+    k_pr_init_edges<<<gs * 2, 256, 0, s>>>(p.row_ptr, p.col, res, (uint32_t)n, (uint32_t)p.m_local,
+                                            (1.0 - alpha) * alpha);
+    g_launches++;
+  }
+  k_pr_seed<<<gs, 1024, 0, s>>>(res, n, eps, q, r.watchdog_ns);
+  g_launches++;
+  ATOS_CUDA(cudaGetLastError());
+  if (r.l2_persist) set_l2_window(s, res, (size_t)n * 8, true);
+  PrApp app{p.row_ptr, p.col, rank, res, alpha, eps, r.check_size > 0 ? 0 : 1};
+  p.ring_clean = false;
+  int rc = ATOS_OK;
+  if (r.check_size <= 0) {
+    rc = launch_relax(app, q, r, p, st);
+  } else {
+    // Check_Size variant: activation only by round-robin sweeps of
+    // Check_Size ids.  Drain the queue, sweep all n ids, repeat until a full
+    // sweep enqueues nothing (every residue <= eps).
+    unsigned long long* h = (unsigned long long*)p.host_pinned;
+    for (int iter = 0; iter < 100000 && rc == ATOS_OK; ++iter) {
+      rc = launch_relax(app, q, r, p, st);
+      if (rc != ATOS_OK) break;
+      ATOS_CUDA(cudaMemcpyAsync(h, &q.ctl->tail.v, 8, cudaMemcpyDeviceToHost, s));
+      ATOS_TRY(stream_wait(s, r.timeout_s));
+      const unsigned long long t_before = h[0];
+      ATOS_CUDA(cudaMemsetAsync(&q.ctl->check.v, 0, 8, s));
+      k_pr_sweep<<<gs, 256, 0, s>>>(res, n, eps, q, (uint32_t)r.check_size, r.watchdog_ns);
+      g_launches++;
+      ATOS_CUDA(cudaMemcpyAsync(h, &q.ctl->tail.v, 8, cudaMemcpyDeviceToHost, s));
+      ATOS_TRY(stream_wait(s, r.timeout_s));
+      if (h[0] == t_before) break;
+    }
+  }
+  if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
+  if (rc != ATOS_OK) return rc;
+  ATOS_CUDA(cudaMemsetAsync(sum, 0, 8, s));
+  k_pr_finalize<<<gs, 256, 0, s>>>(rank, res, n, sum);
+  g_launches++;
+  ATOS_CUDA(cudaGetLastError());
+  rc = finish_queue(p, s, st, "pagerank");
+  if (rc != ATOS_OK) return rc;
+  if (st) {
+    double h_sum = 0;
+    ATOS_CUDA(cudaMemcpy(&h_sum, sum, 8, cudaMemcpyDeviceToHost));
+    st->residual_sum = h_sum;
+  }
+  return ATOS_OK;
+}
+
+}  // namespace atos

@@ -1,0 +1,167 @@
+"""GPU parity: atos_bfs (through the C ABI) vs the serial oracle, bit-exact (BASELINE north_star).
+
+Covers the design space of the paper's Queues API (Listing 3):
+worker size thread / warp / CTA, FETCH_SIZE, persistent vs discrete,
+dedupe on/off, at sizes spanning many fetch chunks with ragged tails, plus
+the degenerate cases (isolated source, directed chain, empty rows).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_icpp_chenbpbyo22_b200 as atos
+from paper_conf_icpp_chenbpbyo22_b200 import gen
+
+import _graphs as G
+from _gpu import DEV, as_u32, csr_of
+
+pytestmark = pytest.mark.gpu
+
+KNOBS = [
+    dict(worker=256, fetch_size=256, persistent=1),
+    dict(worker=256, fetch_size=64, persistent=1),
+    dict(worker=128, fetch_size=512, persistent=1),
+    dict(worker=1024, fetch_size=1024, persistent=1),
+    dict(worker=32, fetch_size=1, persistent=1),
+    dict(worker=32, fetch_size=8, persistent=1),
+    dict(worker=1, fetch_size=1, persistent=1),
+    dict(worker=1, fetch_size=4, persistent=1),
+    dict(worker=256, fetch_size=256, persistent=0),
+    dict(worker=32, fetch_size=8, persistent=0),
+    dict(worker=1, fetch_size=2, persistent=0),
+    dict(worker=256, fetch_size=256, persistent=1, dedupe=0),
+    dict(worker=32, fetch_size=4, persistent=1, dedupe=0),
+]
+
+
+def kid(k):
+    return "-".join(f"{a}{b}" for a, b in k.items())
+
+
+@pytest.fixture(scope="module")
+def rmat14():
+    g = gen.rmat(14, 16, seed=7)
+    rp, ci = g.numpy()
+    return rp, ci, atos.CSR.from_graph(g.to(DEV))
+
+
+@pytest.mark.parametrize("knobs", KNOBS, ids=kid)
+def test_rmat_all_knobs(rmat14, knobs):
+    rp, ci, csr = rmat14
+    for s in (gen.pick_source(gen.Graph(len(rp) - 1, len(ci), torch.from_numpy(rp), torch.from_numpy(ci)), 3), 0, 1):
+        d, st = atos.bfs(csr, s, **knobs)
+        want = oracle.bfs(rp, ci, s)
+        np.testing.assert_array_equal(as_u32(d), want)
+        reached = int(np.sum(want != 0xFFFFFFFF))
+        assert st["pops"] >= reached  # every reached vertex expanded at least once
+
+
+@pytest.mark.parametrize("knobs", KNOBS[:1] + KNOBS[4:5] + KNOBS[8:9] + KNOBS[6:7], ids=kid)
+def test_mesh_closed_form(knobs):
+    R, C = 300, 257
+    g = gen.mesh(R, C)
+    csr = atos.CSR.from_graph(g.to(DEV))
+    r, c = np.divmod(np.arange(R * C), C)
+    for (r0, c0) in ((0, 0), (R // 2, C // 2), (R - 1, 5)):
+        d, st = atos.bfs(csr, r0 * C + c0, **knobs)
+        np.testing.assert_array_equal(as_u32(d), np.abs(r - r0) + np.abs(c - c0))
+
+
+def test_mesh_road_percolated():
+    g = gen.mesh(200, 200, keep_prob=0.6, seed=2)
+    rp, ci = g.numpy()
+    csr = atos.CSR.from_graph(g.to(DEV))
+    src = gen.mesh_centre_source(g, 200, 200)
+    for knobs in (KNOBS[0], KNOBS[8], KNOBS[4]):
+        d, _ = atos.bfs(csr, src, **knobs)
+        np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, src))
+
+
+@pytest.mark.parametrize("name", ["path", "star", "disconnected", "dchain", "complete", "single_edge"])
+def test_small_named(name):
+    rp, ci = {
+        "path": G.path(1000), "star": G.star(3000), "complete": G.complete(40),
+        "disconnected": G.csr_from_edges(50, [(0, 1), (1, 2), (10, 11)], symmetric=True),
+        "dchain": G.csr_from_edges(6, [(0, 1), (1, 2), (2, 3), (3, 4), (4, 5)]),
+        "single_edge": G.csr_from_edges(2, [(0, 1)]),
+    }[name]
+    n = len(rp) - 1
+    csr = csr_of(rp, ci)
+    for knobs in KNOBS:
+        for s in sorted({0, n - 1, n // 2}):
+            d, _ = atos.bfs(csr, s, **knobs)
+            np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, s), err_msg=f"{name} s={s} {knobs}")
+
+
+def test_isolated_source():
+    rp, ci = G.csr_from_edges(10, [(1, 2), (2, 3)], symmetric=True)
+    csr = csr_of(rp, ci)
+    d, st = atos.bfs(csr, 0)
+    want = np.full(10, 0xFFFFFFFF, dtype=np.uint32)
+    want[0] = 0
+    np.testing.assert_array_equal(as_u32(d), want)
+    assert st["pops"] == 1
+
+
+def test_host_input_and_output():
+    g = gen.rmat(12, 8, seed=3)
+    rp, ci = g.numpy()
+    csr = csr_of(rp, ci, host=True)
+    out = torch.empty(g.n, dtype=torch.int32).pin_memory()
+    s = gen.pick_source(g, 1)
+    d, _ = atos.bfs(csr, s, out=out)
+    assert not d.is_cuda
+    np.testing.assert_array_equal(d.numpy().view(np.uint32), oracle.bfs(rp, ci, s))
+
+
+def test_repeat_calls_reuse_workspace():
+    g = gen.rmat(13, 16, seed=5)
+    rp, ci = g.numpy()
+    csr = atos.CSR.from_graph(g.to(DEV))
+    for s in range(0, 200, 17):
+        d, _ = atos.bfs(csr, s)
+        np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, s))
+
+
+def test_errors():
+    g = gen.rmat(8, 4, seed=1)
+    csr = atos.CSR.from_graph(g.to(DEV))
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.bfs(csr, g.n)
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.bfs(csr, 0, worker=48)
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.bfs(csr, 0, fetch_size=0, worker=5)
+    bad_rp = torch.tensor([0, 2, 1], dtype=torch.int64, device=DEV)
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.CSR(bad_rp, torch.tensor([1, 0], dtype=torch.int32, device=DEV))
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.CSR(torch.tensor([0, 1], dtype=torch.int64), torch.tensor([5], dtype=torch.int32))
+
+
+def test_small_queue_overflow_reports_error():
+    # paper-literal (dedupe=0) with a tiny ring must fail loudly, never hang
+    g = gen.rmat(12, 16, seed=2)
+    csr = atos.CSR.from_graph(g.to(DEV))
+    try:
+        atos.bfs(csr, gen.pick_source(g, 1), dedupe=0, queue_capacity=64, timeout_s=2.0)
+    except RuntimeError as e:
+        assert "OVERFLOW" in str(e) or "TIMEOUT" in str(e)
+    # the handle stays usable afterwards
+    rp, ci = g.numpy()
+    d, _ = atos.bfs(csr, 0)
+    np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, 0))
+
+
+@pytest.mark.slow
+def test_config_c1_bench_launch():
+    """C1 (RMAT S16 EF16, seed 1, source seed 101) at the bench's launch configuration."""
+    g = gen.make_config("C1", device=DEV)
+    rp, ci = g.numpy()
+    csr = atos.CSR.from_graph(g)
+    src = gen.pick_source(g, 101)
+    want = oracle.bfs(rp, ci, src)
+    for knobs in (dict(), dict(worker=32), dict(persistent=0)):
+        d, st = atos.bfs(csr, src, **knobs)
+        np.testing.assert_array_equal(as_u32(d), want)
