@@ -96,20 +96,35 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
   }
   r->stream = (cudaStream_t)d.stream;
   r->stats = d.stats;
-  r->watchdog_ns = (unsigned long long)((r->timeout_s > 0 ? r->timeout_s : 30.0) * 1e9);
+  r->watchdog_ns = (unsigned long long)((r->timeout_s > 0 ? r->timeout_s : 10.0) * 1e9);
   return ATOS_OK;
+}
+
+// Fresh ring: slot i free for index i (seq = i), all counters 0.
+__global__ void k_ring_init(unsigned long long* slots, unsigned long long cap, QueueCtl* ctl) {
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < cap;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    slots[i] = make_slot(i, 0u);
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    ctl->head.v = 0;
+    ctl->tail.v = 0;
+    ctl->done.v = 0;
+    ctl->status.v = 0;
+  }
 }
 
 int ensure_queue(Part& p, uint64_t cap, cudaStream_t s) {
   if (p.ring_cap < cap || !p.ring.p) {
-    ATOS_TRY(p.ring.ensure(cap * 4));
+    ATOS_TRY(p.ring.ensure(cap * 8));
     p.ring_cap = cap;
     p.ring_clean = false;
   }
   if (!p.ctl.p) ATOS_TRY(p.ctl.ensure(sizeof(QueueCtl)));
   if (!p.host_pinned) ATOS_CUDA(cudaHostAlloc(&p.host_pinned, 4096, cudaHostAllocDefault));
   if (!p.ring_clean) {
-    ATOS_CUDA(cudaMemsetAsync(p.ring.p, 0xFF, p.ring_cap * 4, s));
+    k_ring_init<<<1184, 256, 0, s>>>(p.ring.as<unsigned long long>(), p.ring_cap, p.ctl.as<QueueCtl>());
+    g_launches++;
+    ATOS_CUDA(cudaGetLastError());
     p.ring_clean = true;
   }
   return ATOS_OK;

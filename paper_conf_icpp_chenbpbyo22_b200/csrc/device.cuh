@@ -3,14 +3,21 @@
 //
 // Queue design (ours; the paper specifies only "concurrent_pop / concurrent_push"
 // on a single shared queue, and push_warp):
-//   * ring u32 items[C], C a power of two, every slot EMPTY (0xFFFFFFFF) when idle;
+//   * ring of C 64-bit slots (C a power of two), slot = (seq << 32) | item,
+//     a per-slot sequence number in the style of Vyukov's bounded MPMC queue:
+//       slot idx&mask is free for the producer of index idx  iff seq == idx,
+//       it holds the item of index idx                         iff seq == idx+1,
+//     (seq compared modulo 2^32);
 //   * 64-bit monotone counters head (claims), tail (reservations), done
-//     (completed tasks), each on its own 128-byte line -- they never wrap, so
-//     there is no ABA;
-//   * a producer reserves [t, t+k) with ONE atomicAdd per warp-batch, writes the
-//     ids with st.release (publication); a consumer claims [h, h+k) with ONE
-//     atomicAdd per worker, spins on ld.acquire until a slot != EMPTY, takes
-//     the id and stores EMPTY back;
+//     (completed tasks), each on its own 128-byte line; they persist across
+//     runs (a run starts with head = done = tail), so the ring never needs
+//     re-initialisation between calls;
+//   * a producer reserves [t, t+k) with ONE atomicAdd per warp-batch and
+//     publishes each slot with one st.release of (idx+1, item); a consumer
+//     claims [h, h+k) with ONE atomicAdd per worker, waits (without blocking
+//     its ready work) for seq == idx+1, takes the item and frees the slot for
+//     the next lap with seq = idx + C.  Over-claimed indices (>= tail) are
+//     therefore never confused with another lap's item;
 //   * termination: done == tail read after an acquire of done (DESIGN.md
 //     "Termination"): every reserved slot has been processed, so no task is in
 //     flight and none can be produced.
@@ -47,10 +54,14 @@ struct QueueCtl {
 };
 
 struct Ring {
-  uint32_t* items;
-  unsigned long long mask;  // C - 1
+  unsigned long long* slots;  // C slots of (seq << 32 | item)
+  unsigned long long mask;    // C - 1
   QueueCtl* ctl;
 };
+
+__device__ __forceinline__ unsigned long long make_slot(unsigned long long seq, uint32_t item) {
+  return ((unsigned long long)(uint32_t)seq << 32) | item;
+}
 
 // ---------------------------------------------------------------- memory order
 __device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
@@ -82,6 +93,12 @@ __device__ __forceinline__ unsigned long long ld_acquire(const unsigned long lon
   unsigned long long v;
   asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
+}
+__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
@@ -137,6 +154,36 @@ __device__ __forceinline__ unsigned long long splitmix64(unsigned long long x) {
 }
 
 // -------------------------------------------------------------------- pushing
+// Publish `item` at reserved index idx: wait (bounded) until the slot is free
+// for this lap, then one release store of (idx+1, item).
+__device__ __forceinline__ void publish_one(const Ring& q, unsigned long long idx, uint32_t item,
+                                            unsigned long long watchdog_ns) {
+  unsigned long long* slot = q.slots + (idx & q.mask);
+  if ((uint32_t)(ld_relaxed(slot) >> 32) != (uint32_t)idx) {
+    // the previous lap's item in this slot has not been consumed yet: wait, bounded
+    unsigned long long t0 = globaltimer();
+    while ((uint32_t)(ld_relaxed(slot) >> 32) != (uint32_t)idx) {
+      __nanosleep(256);
+      if (globaltimer() - t0 > watchdog_ns) {
+        atomicOr((unsigned int*)&q.ctl->status.v, kStatusOverflow);
+        return;
+      }
+    }
+  }
+  st_release(slot, make_slot(idx + 1, item));
+}
+
+// Try to take the item of index idx: true + *item on success (slot freed for the next lap).
+__device__ __forceinline__ bool try_consume(const Ring& q, unsigned long long idx, uint32_t* item) {
+  unsigned long long* slot = q.slots + (idx & q.mask);
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(slot) : "memory");
+  if ((uint32_t)(v >> 32) != (uint32_t)(idx + 1)) return false;
+  *item = (uint32_t)v;
+  st_relaxed(slot, make_slot(idx + q.mask + 1, 0u));
+  return true;
+}
+
 // Per-warp staging buffer in shared memory.  push() is warp-collective (all 32
 // lanes call it with their own `want` flag); entries accumulate and are
 // published 32 at a time: one atomicAdd on tail per 32 pushes, one coalesced
@@ -151,21 +198,7 @@ struct WarpPusher {
     unsigned long long base = 0;
     if (lane_id() == 0) base = atomicAdd(&q.ctl->tail.v, (unsigned long long)k);
     base = __shfl_sync(0xffffffffu, base, 0);
-    if (lane_id() < k) {
-      uint32_t* slot = q.items + ((base + lane_id()) & q.mask);
-      if (ld_relaxed(slot) != kEmpty) {
-        // ring lapped a slot that has not been consumed yet: wait, bounded
-        unsigned long long t0 = globaltimer();
-        while (ld_relaxed(slot) != kEmpty) {
-          __nanosleep(256);
-          if (globaltimer() - t0 > watchdog_ns) {
-            atomicOr((unsigned int*)&q.ctl->status.v, kStatusOverflow);
-            break;
-          }
-        }
-      }
-      st_release(slot, buf[lane_id()]);
-    }
+    if (lane_id() < k) publish_one(q, base + lane_id(), buf[lane_id()], watchdog_ns);
     total += k;
   }
 

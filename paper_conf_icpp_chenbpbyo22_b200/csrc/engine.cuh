@@ -90,101 +90,112 @@ __device__ __forceinline__ uint32_t group_size() {
   return MODE == MODE_CTA ? blockDim.x : 32u;
 }
 
-// Try to consume slot `idx`: on success the item goes to s.item[] and the slot
-// is reset to EMPTY; otherwise idx is appended to the new pending list.
+// Try to consume index `idx`: on success the item goes to s.item[] (slot freed
+// for the next lap); otherwise idx is appended to the new pending list.
 template <class Payload>
 __device__ __forceinline__ void consume_slot(const Ring& q, const GroupSmem<Payload>& s,
                                              unsigned long long idx) {
-  uint32_t* slot = q.items + (idx & q.mask);
-  uint32_t v = ld_acquire(slot);
-  if (v == kEmpty) {
+  uint32_t v;
+  if (!try_consume(q, idx, &v)) {
     uint32_t k = atomicAdd(&s.ctr[2], 1u);
     s.pend2[k] = idx;
   } else {
-    st_relaxed(slot, kEmpty);
     uint32_t k = atomicAdd(&s.ctr[0], 1u);
     s.item[k] = v;
   }
 }
 
-// ------------------------------------------------------------------- kernel
-template <class App, int MODE, bool PERSIST>
-__global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) {
-  using Payload = typename App::Payload;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  const uint32_t nwarps = blockDim.x >> 5;
-  const uint32_t K = (MODE == MODE_THREAD) ? 32u * P.fetch : P.fetch;
-  const size_t gbytes = group_smem_bytes<Payload>(K);
-  // push buffers first (64 u32 per warp), then one arena per group
-  uint32_t* pushbuf = (uint32_t*)smem_raw;
-  unsigned char* arena = smem_raw + (size_t)nwarps * 64 * 4;
-  const uint32_t gid = (MODE == MODE_CTA) ? 0 : warp_id();
-  GroupSmem<Payload> s = carve<Payload>(arena + gbytes * gid, K);
-  const uint32_t r = group_rank<MODE>(), G = group_size<MODE>();
+// ------------------------------------------------------------ worker group
+// One worker (a CTA, a warp, or -- for MODE_THREAD -- a warp of 32 thread
+// workers that share one claim) and its queue protocol: claim / gather /
+// idle-with-termination (acquire) and completion (complete).
+template <int MODE, bool PERSIST, class Payload>
+struct Worker {
+  GroupSmem<Payload> s;
+  uint32_t r, G, K;
+  unsigned long long ggid;
+  bool first;
+  unsigned backoff;
+  unsigned long long idle_since;
 
-  WarpPusher pusher{pushbuf + warp_id() * 64, 0, 0};
-  unsigned long long my_pops = 0, my_edges = 0;
-  const Ring& q = P.q;
+  __device__ __forceinline__ void init(unsigned char* arena, const EngineParams& P) {
+    const uint32_t nwarps = blockDim.x >> 5;
+    K = (MODE == MODE_THREAD) ? 32u * P.fetch : P.fetch;
+    const uint32_t gid = (MODE == MODE_CTA) ? 0 : warp_id();
+    s = carve<Payload>(arena + group_smem_bytes<Payload>(K) * gid, K);
+    r = group_rank<MODE>();
+    G = group_size<MODE>();
+    const unsigned long long groups_per_block = (MODE == MODE_CTA) ? 1 : nwarps;
+    ggid = (unsigned long long)blockIdx.x * groups_per_block + gid;
+    first = true;
+    backoff = 32;
+    idle_since = 0;
+    if (r == 0) s.ctr[1] = 0;
+    group_sync<MODE>();
+  }
 
-  // group index across the grid (discrete mode static chunking)
-  const unsigned long long groups_per_block = (MODE == MODE_CTA) ? 1 : nwarps;
-  const unsigned long long ggid = (unsigned long long)blockIdx.x * groups_per_block + gid;
-
-  if (r == 0) { s.ctr[1] = 0; }
-  group_sync<MODE>();
-
-  bool first = true;
-  unsigned backoff = 32;
-  unsigned long long idle_since = 0;
-  while (true) {
-    // ---------------------------------------------------------- 1. claim
-    if (r == 0) {
-      s.ctr[0] = 0; s.ctr[2] = 0; s.ctr[3] = 0; s.ctr[4] = 0;
-      *(unsigned long long*)&s.ctr[6] = 0;
-      if (!PERSIST) {
-        if (!first) {
-          s.ctr[3] = 1;
-        } else {
-          unsigned long long b = P.h0 + ggid * K;
-          unsigned long long e = b + K < P.t0 ? b + K : P.t0;
-          if (b >= P.t0) s.ctr[3] = 1;
-          else { *(unsigned long long*)&s.ctr[6] = b; s.ctr[4] = (uint32_t)(e - b); }
-        }
-      } else if (s.ctr[1] == 0) {
-        unsigned long long h = ld_relaxed(&q.ctl->head.v);
-        unsigned long long t = ld_relaxed(&q.ctl->tail.v);
-        if (h < t) {
-          unsigned long long amt = t - h < K ? t - h : K;
-          unsigned long long b = atomicAdd(&q.ctl->head.v, amt);
-          *(unsigned long long*)&s.ctr[6] = b;
-          s.ctr[4] = (uint32_t)amt;
+  // Returns the number of ready items now in s.item[0..n), or 0 when the
+  // worker must exit (global termination, watchdog, or end of a discrete chunk).
+  __device__ __forceinline__ uint32_t acquire(const EngineParams& P) {
+    const Ring& q = P.q;
+    while (true) {
+      // ------------------------------------------------------ 1. claim
+      if (r == 0) {
+        s.ctr[0] = 0; s.ctr[2] = 0; s.ctr[3] = 0; s.ctr[4] = 0;
+        *(unsigned long long*)&s.ctr[6] = 0;
+        if (!PERSIST) {
+          if (!first) {
+            s.ctr[3] = 1;
+          } else {
+            const unsigned long long b = P.h0 + ggid * K;
+            const unsigned long long e = b + K < P.t0 ? b + K : P.t0;
+            if (b >= P.t0) s.ctr[3] = 1;
+            else { *(unsigned long long*)&s.ctr[6] = b; s.ctr[4] = (uint32_t)(e - b); }
+          }
+        } else if (s.ctr[1] == 0) {
+          // bounded over-claim: at most the items visible at the tail
+          const unsigned long long h = ld_relaxed(&q.ctl->head.v);
+          const unsigned long long t = ld_relaxed(&q.ctl->tail.v);
+          if (h < t) {
+            const unsigned long long amt = t - h < K ? t - h : K;
+            const unsigned long long b = atomicAdd(&q.ctl->head.v, amt);
+            *(unsigned long long*)&s.ctr[6] = b;
+            s.ctr[4] = (uint32_t)amt;
+          }
         }
       }
-    }
-    first = false;
-    group_sync<MODE>();
-    if (s.ctr[3]) break;
-    // ---------------------------------------------------------- 2. gather
-    {
-      const unsigned long long cb = *(unsigned long long*)&s.ctr[6];
-      const uint32_t cc = s.ctr[4], np = s.ctr[1];
-      for (uint32_t i = r; i < cc; i += G) consume_slot(q, s, cb + i);
-      for (uint32_t i = r; i < np; i += G) consume_slot(q, s, s.pend[i]);
-    }
-    group_sync<MODE>();
-    const uint32_t nready = s.ctr[0];
-    if (nready == 0) {
-      // nothing ready: idle path (f2 in Listing 3) -- termination check + backoff
+      first = false;
+      group_sync<MODE>();
+      if (s.ctr[3]) return 0;
+      // ------------------------------------------------------ 2. gather
+      {
+        const unsigned long long cb = *(unsigned long long*)&s.ctr[6];
+        const uint32_t cc = s.ctr[4], np = s.ctr[1];
+        for (uint32_t i = r; i < cc; i += G) consume_slot(q, s, cb + i);
+        for (uint32_t i = r; i < np; i += G) consume_slot(q, s, s.pend[i]);
+      }
+      group_sync<MODE>();
+      const uint32_t nready = s.ctr[0];
+      const uint32_t npn = s.ctr[2];
+      for (uint32_t i = r; i < npn; i += G) s.pend[i] = s.pend2[i];
+      group_sync<MODE>();
+      if (nready) {
+        if (r == 0) s.ctr[1] = npn;
+        idle_since = 0;
+        backoff = 32;
+        group_sync<MODE>();
+        return nready;
+      }
+      // ------------------------------------------------------ 3. idle (f2)
       if (r == 0) {
-        // move pending list
-        s.ctr[1] = s.ctr[2];
-        for (uint32_t i = 0; i < s.ctr[2]; ++i) s.pend[i] = s.pend2[i];
-        unsigned long long d = atom_read(&q.ctl->done.v);
-        unsigned long long t = atom_read(&q.ctl->tail.v);
-        uint32_t st = *(volatile uint32_t*)&q.ctl->status.v;
-        if (d == t || st != 0) s.ctr[3] = 1;
-        else {
-          unsigned long long now = globaltimer();
+        s.ctr[1] = npn;
+        const unsigned long long d = atom_read(&q.ctl->done.v);
+        const unsigned long long t = atom_read(&q.ctl->tail.v);
+        const uint32_t st = *(volatile uint32_t*)&q.ctl->status.v;
+        if (d == t || st != 0) {
+          s.ctr[3] = 1;
+        } else {
+          const unsigned long long now = globaltimer();
           if (idle_since == 0) idle_since = now;
           else if (now - idle_since > P.watchdog_ns) {
             atomicOr((unsigned int*)&q.ctl->status.v, kStatusTimeout);
@@ -195,17 +206,55 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
         }
       }
       group_sync<MODE>();
-      if (s.ctr[3]) break;
-      continue;
+      if (s.ctr[3]) return 0;
     }
-    idle_since = 0;
-    backoff = 32;
-    // pending list for the next iteration (copied in parallel)
-    {
-      const uint32_t npn = s.ctr[2];
-      for (uint32_t i = r; i < npn; i += G) s.pend[i] = s.pend2[i];
+  }
+
+  // All pushes of the batch are published (every warp flushed before this):
+  // count the batch as done with release semantics.
+  __device__ __forceinline__ void complete(const EngineParams& P, uint32_t nready) {
+    group_sync<MODE>();
+    if (PERSIST && r == 0) {
+      fence_acq_rel_gpu();
+      atom_add_release(&P.q.ctl->done.v, (unsigned long long)nready);
     }
-    // ---------------------------------------------------------- 3. begin (per item)
+    group_sync<MODE>();
+  }
+};
+
+__device__ __forceinline__ void flush_stats(const Ring& q, unsigned long long pops, unsigned long long edges,
+                                            unsigned long long pushes_lane0) {
+  for (int o = 16; o; o >>= 1) {
+    pops += __shfl_xor_sync(0xffffffffu, pops, o);
+    edges += __shfl_xor_sync(0xffffffffu, edges, o);
+  }
+  if (lane_id() == 0) {
+    if (pops) atomicAdd(&q.ctl->stat_pops.v, pops);
+    if (edges) atomicAdd(&q.ctl->stat_edges.v, edges);
+    if (pushes_lane0) atomicAdd(&q.ctl->stat_pushes.v, pushes_lane0);
+  }
+}
+
+// ------------------------------------------------------------------- kernel
+template <class App, int MODE, bool PERSIST>
+__global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) {
+  using Payload = typename App::Payload;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const uint32_t nwarps = blockDim.x >> 5;
+  // push buffers first (64 u32 per warp), then one arena per group
+  uint32_t* pushbuf = (uint32_t*)smem_raw;
+  Worker<MODE, PERSIST, Payload> wk;
+  wk.init(smem_raw + (size_t)nwarps * 64 * 4, P);
+  const GroupSmem<Payload>& s = wk.s;
+  const uint32_t r = wk.r, G = wk.G;
+  WarpPusher pusher{pushbuf + warp_id() * 64, 0, 0};
+  unsigned long long my_pops = 0, my_edges = 0;
+  const Ring& q = P.q;
+
+  while (true) {
+    const uint32_t nready = wk.acquire(P);
+    if (nready == 0) break;
+    // ---------------------------------------------------------- begin (per item)
     for (uint32_t k = r; k < nready; k += G) {
       uint32_t st = 0, dg = 0;
       Payload p{};
@@ -215,20 +264,18 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
       s.pay[k] = p;
     }
     group_sync<MODE>();
-    if (r == 0) s.ctr[1] = s.ctr[2];
     my_pops += (r == 0) ? nready : 0;
 
-    // ---------------------------------------------------------- 4. expand + relax
+    // ---------------------------------------------------------- expand + relax
     if (MODE == MODE_CTA) {
       // load-balancing search over the flattened edge list of the batch
       uint32_t total = 0;
       uint32_t mydeg = 0;
-      // scan: each thread owns ceil(nready/B) consecutive items
       const uint32_t per = (nready + G - 1) / G;
-      const uint32_t i0 = r * per, i1 = min(i0 + per, nready);
+      const uint32_t i0 = min(r * per, nready), i1 = min(i0 + per, nready);
       for (uint32_t i = i0; i < i1; ++i) mydeg += s.off[i];
       uint32_t excl = block_exclusive_scan(mydeg, s.ctr + 8, &total);
-      for (uint32_t i = i0; i < i1; ++i) { uint32_t d = s.off[i]; s.off[i] = excl; excl += d; }
+      for (uint32_t i = i0; i < i1; ++i) { const uint32_t d = s.off[i]; s.off[i] = excl; excl += d; }
       __syncthreads();
       my_edges += (r == 0) ? total : 0;
       for (uint32_t base = 0; base < total; base += G) {
@@ -239,7 +286,7 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
           // largest i with off[i] <= e
           uint32_t lo = 0, hi = nready;
           while (hi - lo > 1) {
-            uint32_t mid = (lo + hi) >> 1;
+            const uint32_t mid = (lo + hi) >> 1;
             if (s.off[mid] <= e) lo = mid; else hi = mid;
           }
           const uint32_t w = __ldg(app.col + s.start[lo] + (e - s.off[lo]));
@@ -287,26 +334,9 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
       }
     }
     pusher.flush(q, P.watchdog_ns);
-    // ---------------------------------------------------------- 5. complete
-    group_sync<MODE>();
-    if (PERSIST && r == 0) {
-      // release: this group's pushes (tail reservations + slot stores) happen-before done
-      fence_acq_rel_gpu();
-      atom_add_release(&q.ctl->done.v, (unsigned long long)nready);
-    }
-    group_sync<MODE>();
+    wk.complete(P, nready);
   }
-  // statistics: one atomic per warp
-  unsigned long long pushes = lane_id() == 0 ? pusher.total : 0;
-  for (int o = 16; o; o >>= 1) {
-    my_pops += __shfl_xor_sync(0xffffffffu, my_pops, o);
-    my_edges += __shfl_xor_sync(0xffffffffu, my_edges, o);
-  }
-  if (lane_id() == 0) {
-    atomicAdd(&q.ctl->stat_pops.v, my_pops);
-    atomicAdd(&q.ctl->stat_edges.v, my_edges);
-    atomicAdd(&q.ctl->stat_pushes.v, pushes);
-  }
+  flush_stats(q, my_pops, my_edges, lane_id() == 0 ? pusher.total : 0);
 }
 
 // Host-side helper: dynamic shared memory for a launch.

@@ -8,36 +8,40 @@
 namespace atos {
 
 // ------------------------------------------------------------- init kernels
-// BFS init (Alg.1 P:721-725 "vertex.dist = MAX_UINT32", frontier = [source];
-// source depth 0, R-BFS-1).  depth[] was memset to 0xFF on the stream.
-__global__ void k_bfs_init(uint32_t* depth, uint32_t* inq, uint32_t* ring, QueueCtl* ctl, uint32_t src) {
-  if (threadIdx.x == 0) {
-    depth[src] = 0;
-    if (inq) inq[src >> 5] |= 1u << (src & 31);
-    ring[0] = src;
-    ctl->head.v = 0;
-    ctl->tail.v = 1;
-    ctl->done.v = 0;
-    ctl->status.v = 0;
-    ctl->check.v = 0;
-    ctl->stat_pops.v = 0;
-    ctl->stat_pushes.v = 0;
-    ctl->stat_edges.v = 0;
-    ctl->misc.v = 0;
-  }
+// Start of a run on a persistent ring: abandon stale over-claims (head = tail),
+// done = tail, clear status and per-run statistics.
+__device__ __forceinline__ void run_begin(QueueCtl* ctl) {
+  const unsigned long long t = ctl->tail.v;
+  ctl->head.v = t;
+  ctl->done.v = t;
+  ctl->status.v = 0;
+  ctl->check.v = 0;
+  ctl->stat_pops.v = 0;
+  ctl->stat_pushes.v = 0;
+  ctl->stat_edges.v = 0;
+  ctl->misc.v = 0;
 }
 
-__global__ void k_ctl_reset(QueueCtl* ctl) {
-  if (threadIdx.x == 0) {
-    ctl->head.v = 0;
-    ctl->tail.v = 0;
-    ctl->done.v = 0;
-    ctl->status.v = 0;
-    ctl->check.v = 0;
-    ctl->stat_pops.v = 0;
-    ctl->stat_pushes.v = 0;
-    ctl->stat_edges.v = 0;
-    ctl->misc.v = 0;
+// Before every persistent launch: over-claims abandoned by a previous kernel
+// of the same run are dropped (nothing is in flight between launches).
+__global__ void k_sync_head(QueueCtl* ctl) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) ctl->head.v = ctl->tail.v;
+}
+
+__global__ void k_run_begin(QueueCtl* ctl) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) run_begin(ctl);
+}
+
+// BFS init (Alg.1 P:721-725 "vertex.dist = MAX_UINT32", frontier = [source];
+// source depth 0, R-BFS-1).  depth[] was memset to 0xFF on the stream.
+__global__ void k_bfs_init(uint32_t* depth, uint32_t* inq, Ring q, uint32_t src, unsigned long long wd) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    run_begin(q.ctl);
+    depth[src] = 0;
+    if (inq) inq[src >> 5] |= 1u << (src & 31);
+    const unsigned long long idx = q.ctl->tail.v;
+    q.ctl->tail.v = idx + 1;
+    publish_one(q, idx, src, wd);
   }
 }
 
@@ -158,6 +162,8 @@ static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, 
     int grid = 0;
     ATOS_TRY(persistent_grid(fn, block, smem, &grid));
     if (r.num_blocks > 0) grid = std::min(grid, r.num_blocks);
+    k_sync_head<<<1, 32, 0, s>>>(P.q.ctl);
+    g_launches++;
     void* args[] = {(void*)&app, (void*)&P};
     ATOS_CUDA(cudaLaunchCooperativeKernel(fn, grid, block, args, smem, s));
     g_launches++;
@@ -173,9 +179,10 @@ static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, 
   const uint64_t items_per_block = K * groups_per_block;
   unsigned long long* h_ctl = (unsigned long long*)p.host_pinned;
   QueueCtl* ctl = P.q.ctl;
-  ATOS_CUDA(cudaMemcpyAsync(h_ctl, &ctl->tail.v, 8, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaMemcpyAsync(h_ctl, &ctl->head.v, 16 * 8 * 2, cudaMemcpyDeviceToHost, s));
   ATOS_CUDA(cudaStreamSynchronize(s));
-  uint64_t h0 = 0, t0 = h_ctl[0];
+  // head line then tail line (Line64 = 16 words)
+  uint64_t h0 = h_ctl[0], t0 = h_ctl[16];
   // the discrete frontier is consumed in order, so head follows h0
   while (h0 < t0) {
     P.h0 = h0;
@@ -219,7 +226,7 @@ static int launch_relax(const App& app, const Ring& q, const Resolved& r, Part& 
 
 static Ring ring_of(Part& p) {
   Ring q;
-  q.items = p.ring.as<uint32_t>();
+  q.slots = p.ring.as<unsigned long long>();
   q.mask = p.ring_cap - 1;
   q.ctl = p.ctl.as<QueueCtl>();
   return q;
@@ -240,7 +247,7 @@ int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolve
   }
   ATOS_CUDA(cudaMemsetAsync(depth, 0xFF, (size_t)n * 4, s));
   Ring q = ring_of(p);
-  k_bfs_init<<<1, 32, 0, s>>>(depth, inq, q.items, q.ctl, (uint32_t)src);
+  k_bfs_init<<<1, 32, 0, s>>>(depth, inq, q, (uint32_t)src, r.watchdog_ns);
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, depth, (size_t)n * 4, true);
@@ -264,7 +271,7 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
   double* res = p.vbuf_a.as<double>();
   double* sum = p.scratch.as<double>();
   Ring q = ring_of(p);
-  k_ctl_reset<<<1, 32, 0, s>>>(q.ctl);
+  k_run_begin<<<1, 32, 0, s>>>(q.ctl);
   g_launches++;
   const int gs = 148 * 8;
   k_pr_init_vertices<<<gs, 256, 0, s>>>(rank, res, n, 1.0 - alpha);
@@ -292,7 +299,9 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
       rc = launch_relax(app, q, r, p, st);
       if (rc != ATOS_OK) break;
       ATOS_CUDA(cudaMemcpyAsync(h, &q.ctl->tail.v, 8, cudaMemcpyDeviceToHost, s));
+      ATOS_CUDA(cudaMemcpyAsync(h + 1, &q.ctl->status.v, 8, cudaMemcpyDeviceToHost, s));
       ATOS_TRY(stream_wait(s, r.timeout_s));
+      if (h[1] != 0) break;  // watchdog/overflow: reported by finish_queue
       const unsigned long long t_before = h[0];
       ATOS_CUDA(cudaMemsetAsync(&q.ctl->check.v, 0, 8, s));
       k_pr_sweep<<<gs, 256, 0, s>>>(res, n, eps, q, (uint32_t)r.check_size, r.watchdog_ns);
