@@ -1,0 +1,409 @@
+#!/usr/bin/env python
+"""Benchmark of the Atos hot path on B200 (BASELINE.json metric:
+"BFS GTEPS, PageRank/colouring ms to converge; % HBM roofline @1/2/4/8 B200").
+
+One STEP = one atos_bfs call (init, persistent worker loop, output; plus the
+exchange rounds at N > 1) from one of 8 seeded sources on the C5 workload
+(RMAT scale 26, edge factor 16, seed 5, 1D vertex-partitioned over N GPUs).
+`value` = whole-job GTEPS = sum over steps of the directed CSR edges of the
+reached vertices (Gunrock convention) / device time.
+PageRank (C3) and colouring (C4) ms-to-converge are reported alongside under
+"apps" (rank 0, N = 1).  Rank 0 prints one JSON line.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl atos|reference]
+                  [--scale S] [--no-apps] [--full]
+
+--impl reference runs the paper-method oracle (oracle/, serial C) on the same
+workload on the host cores (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "BFS GTEPS, PageRank/colouring ms to converge; % HBM roofline @1/2/4/8 B200"
+BFS_BYTES_PER_VERTEX = 20   # row pair 8 + depth[v] 4 + queue write+read 8
+BFS_BYTES_PER_EDGE = 8      # col 4 + depth[w] 4
+PR_BYTES_PER_POP = 32       # row 8 + exch 8 + rank red 8 + queue 8
+PR_BYTES_PER_EDGE = 12      # col 4 + f64 residue RMW 8
+GC_BYTES_PER_TASK = 20      # row 8 + colour 4 + queue 8
+GC_BYTES_PER_EDGE = 8       # col 4 + colour 4
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+def profile_traffic(kernel_key: str):
+    """dram bytes per launch from the committed ncu --set full summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        v = d.get(kernel_key)
+        if isinstance(v, dict):
+            return v.get("dram_bytes_per_launch")
+    return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        self.out = ""
+        if self.proc is not None:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        rows = [r.split(",") for r in (self.out or "").strip().splitlines() if r.count(",") >= 5]
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[0]) for r in rows if r[0].strip().replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].strip().replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if "Active" in r[2 + i] and "Not" not in r[2 + i]})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def dist_setup():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if ws > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    else:
+        torch.cuda.set_device(local)
+    return ws, rank, local
+
+
+def allreduce_max(x: float, ws: int) -> float:
+    if ws == 1:
+        return x
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def allreduce_sum(x: float, ws: int) -> float:
+    if ws == 1:
+        return x
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return float(t.item())
+
+
+def barrier(ws):
+    torch.cuda.synchronize()
+    if ws > 1:
+        import torch.distributed as dist
+        dist.barrier()
+    torch.cuda.synchronize()
+
+
+def flush_l2(buf):
+    buf.zero_()  # 512 MiB write > 126 MB L2
+
+
+def make_graph(scale, ef, seed, device):
+    from paper_conf_icpp_chenbpbyo22_b200 import gen
+    t = time.time()
+    g = gen.rmat(scale, ef, seed, device=device, name=f"rmat-s{scale}-ef{ef}-seed{seed}")
+    torch.cuda.synchronize()
+    log(f"[bench] generated {g.name}: n={g.n} m={g.m} in {time.time() - t:.1f}s")
+    return g
+
+
+def reached_edges(g, depth_i32):
+    deg = g.degrees()
+    reached = depth_i32 != -1
+    return int(reached.sum().item()), int(deg[reached].sum().item())
+
+
+# --------------------------------------------------------------------------- reference arm
+def run_reference(args, ws, rank):
+    """The oracle (serial C, oracle/) timed on the host cores on this workload."""
+    if rank != 0:
+        return
+    import oracle
+    from paper_conf_icpp_chenbpbyo22_b200 import gen
+    g = make_graph(args.scale, 16, 5, "cuda")
+    rp, ci = g.numpy()
+    sources = [gen.pick_source(g, 105 + i) for i in range(8)]
+    del g
+    torch.cuda.empty_cache()
+    times, edges = [], []
+    deg = np.diff(rp)
+    for k in range(args.warmup + args.steps):
+        s = sources[k % len(sources)]
+        t0 = time.perf_counter()
+        d = oracle.bfs(rp, ci, s)
+        dt = time.perf_counter() - t0
+        if k >= args.warmup:
+            times.append(dt)
+            edges.append(int(deg[d != 0xFFFFFFFF].sum()))
+    total = sum(times)
+    value = sum(edges) / total / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": ws,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": total / len(times) * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": f"C5 BFS RMAT scale {args.scale} ef 16 seed 5, 8 seeded sources",
+                   "global_batch": 1, "parallelism": "serial-oracle"},
+        "cpu_baseline": {"value": value, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                         "sample": f"full serial FIFO BFS (oracle_bfs) from each seeded source, {args.steps} steps"},
+        "e2e": {"value": value, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------------------- our arm
+def run_atos(args, ws, rank, local):
+    import paper_conf_icpp_chenbpbyo22_b200 as atos
+    from paper_conf_icpp_chenbpbyo22_b200 import gen
+    dev = torch.device(f"cuda:{local}")
+    peak, peak_kind = measured_peaks()
+    g = make_graph(args.scale, 16, 5, dev)
+    sources = [gen.pick_source(g, 105 + i) for i in range(8)]
+    knobs = dict(worker=args.worker, fetch_size=args.fetch)
+    if ws == 1:
+        csr = atos.CSR.from_graph(g, device=local)
+    else:
+        uid = atos.Comm.unique_id() if rank == 0 else None
+        import torch.distributed as dist
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        comm = atos.Comm(ws, rank, obj[0], local)
+        vb, ve = atos.partition_range(g.n, ws, rank)
+        rp = g.row_ptr[vb:ve + 1] - g.row_ptr[vb]
+        ci = g.col[int(g.row_ptr[vb]):int(g.row_ptr[ve])]
+        csr = comm.partition(g.n, vb, ve, rp.contiguous(), ci.contiguous())
+    # per-source reached vertices / edges (global) for GTEPS and algorithmic bytes
+    out = torch.empty(csr.n_local if ws > 1 else g.n, dtype=torch.int32, device=dev)
+    src_info = []
+    deg_local = g.degrees() if ws == 1 else (g.degrees()[vb:ve])
+    for s in sources:
+        d, st = atos.bfs(csr, s, out=out, **knobs)
+        reached = d != -1
+        nr = allreduce_sum(float(reached.sum().item()), ws)
+        mr = allreduce_sum(float(deg_local[reached].sum().item()), ws)
+        src_info.append((int(nr), int(mr)))
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    for k in range(args.warmup):
+        atos.bfs(csr, sources[k % 8], out=out, **knobs)
+    barrier(ws)
+    times, wtimes, edges, verts = [], [], [], []
+    stream = torch.cuda.current_stream(dev)
+    l0 = atos.launches()
+    with ClockSampler(local) as cs:
+        for k in range(args.steps):
+            flush_l2(flush)
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            _, st = atos.bfs(csr, sources[k % 8], out=out, **knobs)
+            e1.record(stream)
+            e1.synchronize()
+            times.append(e0.elapsed_time(e1))
+            wtimes.append(st["worker_ms"])
+            verts.append(src_info[k % 8][0])
+            edges.append(src_info[k % 8][1])
+    barrier(ws)
+    launches = atos.launches() - l0
+    total_ms = allreduce_max(sum(times), ws)
+    ms_per_step = total_ms / args.steps
+    value = sum(edges) / (total_ms / 1e3) / 1e9
+    clocks = cs.summary()
+    # roofline of the dominant kernel (the persistent BFS worker), algorithmic bytes per launch
+    w_ms = allreduce_max(sum(wtimes), ws) / args.steps
+    alg_bytes = (BFS_BYTES_PER_VERTEX * np.mean(verts) + BFS_BYTES_PER_EDGE * np.mean(edges)) / ws
+    achieved = alg_bytes / (w_ms / 1e3) / 1e9
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": profile_traffic("bfs_worker"), "peak_kind": peak_kind,
+                "kernel": "k_relax_worker<BfsApp,CTA,persistent>", "kernel_ms": w_ms,
+                "worker_share_of_step": w_ms / ms_per_step}
+    line = {
+        "metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak" if ws == 1 else "strong",
+        "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": f"C5: BFS on RMAT scale {args.scale} ef 16 seed 5 (n={g.n}, m={g.m}), "
+                               f"8 seeded sources, 1D vertex partition over {ws} GPU(s)",
+                   "global_batch": 1, "parallelism": f"vertex-partition{ws}", "worker": args.worker,
+                   "fetch_size": args.fetch, "l2": "flushed (512 MiB write) before every timed step",
+                   "mean_reached_vertices": float(np.mean(verts)), "mean_reached_edges": float(np.mean(edges))},
+        "roofline": roofline, "clocks": clocks, "gpu_launches": int(launches),
+    }
+    if rank == 0 and ws == 1:
+        line["e2e"] = e2e_bfs(args, g, sources, src_info, knobs, local)
+        if not args.no_cpu:
+            line["cpu_baseline"] = cpu_baseline(g, sources, src_info)
+        if not args.no_apps:
+            line["apps"] = run_apps(args, dev, peak)
+    elif rank == 0:
+        line["e2e"] = None
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+def e2e_bfs(args, g, sources, src_info, knobs, local, steps=2):
+    """Same metric through the public API with HOST buffers: pinned host CSR -> atos_csr_create
+    (H2D inside the timed region) -> atos_bfs with a host output (D2H) -> destroy."""
+    import paper_conf_icpp_chenbpbyo22_b200 as atos
+    rp_h = g.row_ptr.cpu().pin_memory()
+    ci_h = g.col.cpu().pin_memory()
+    out_h = torch.empty(g.n, dtype=torch.int32).pin_memory()
+    torch.cuda.synchronize()
+    t_total, e_total = 0.0, 0
+    for k in range(steps):
+        t0 = time.perf_counter()
+        csr = atos.CSR(rp_h, ci_h, device=local)
+        atos.bfs(csr, sources[k % 8], out=out_h, **knobs)
+        csr.close()
+        t_total += time.perf_counter() - t0
+        e_total += src_info[k % 8][1]
+    return {"value": e_total / t_total / 1e9, "unit": "GTEPS",
+            "h2d_bytes_per_step": int(rp_h.numel() * 8 + ci_h.numel() * 4),
+            "d2h_bytes_per_step": int(out_h.numel() * 4), "steps": steps,
+            "note": "wall clock around host-synchronous C-ABI calls; includes CSR upload + u32 narrowing"}
+
+
+def cpu_baseline(g, sources, src_info):
+    import oracle
+    rp, ci = g.numpy()
+    t0 = time.perf_counter()
+    d = oracle.bfs(rp, ci, sources[0])
+    dt = time.perf_counter() - t0
+    edges = int(np.diff(rp)[d != 0xFFFFFFFF].sum())
+    return {"value": edges / dt / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+            "sample": f"one full serial FIFO BFS (oracle_bfs, gcc -O2) from source {sources[0]} on the same C5 graph",
+            "seconds": dt}
+
+
+def run_apps(args, dev, peak):
+    """PageRank (C3) and colouring (C4) ms to converge, each with its roofline numbers."""
+    import paper_conf_icpp_chenbpbyo22_b200 as atos
+    res = {}
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    # ---- PageRank on C3
+    g = make_graph(args.pr_scale, 16, 3, dev)
+    csr = atos.CSR.from_graph(g)
+    out = torch.empty(g.n, dtype=torch.float64, device=dev)
+    for _ in range(max(1, args.warmup)):
+        atos.pagerank(csr, 0.85, 1e-6, out=out)
+    ms, wms, pops, edges = [], [], [], []
+    for _ in range(args.app_steps):
+        flush_l2(flush)
+        torch.cuda.synchronize()
+        _, st = atos.pagerank(csr, 0.85, 1e-6, out=out)
+        ms.append(st["kernel_ms"])
+        wms.append(st["worker_ms"])
+        pops.append(st["pops"])
+        edges.append(st["edges"])
+    wm = float(np.mean(wms))
+    alg = PR_BYTES_PER_POP * np.mean(pops) + PR_BYTES_PER_EDGE * np.mean(edges)
+    res["pagerank"] = {"config": f"C3: RMAT scale {args.pr_scale} ef 16 seed 3 (n={g.n}, m={g.m}), alpha 0.85, eps 1e-6",
+                       "ms_to_converge": float(np.mean(ms)), "ms_min": float(np.min(ms)), "worker_ms": wm,
+                       "pops_per_n": float(np.mean(pops)) / g.n, "edge_relaxations_per_m": float(np.mean(edges)) / g.m,
+                       "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
+                       "traffic": profile_traffic("pr_worker")}
+    del csr, g, out
+    torch.cuda.empty_cache()
+    # ---- colouring on C4
+    g = make_graph(args.gc_scale, 64, 4, dev)
+    csr = atos.CSR.from_graph(g)
+    out = torch.empty(g.n, dtype=torch.int32, device=dev)
+    for _ in range(max(1, args.warmup)):
+        atos.color(csr, 1, out=out)
+    ms, wms, pops, edges, cols = [], [], [], [], []
+    for _ in range(args.app_steps):
+        flush_l2(flush)
+        torch.cuda.synchronize()
+        _, st = atos.color(csr, 1, out=out)
+        ms.append(st["kernel_ms"])
+        wms.append(st["worker_ms"])
+        pops.append(st["pops"])
+        edges.append(st["edges"])
+        cols.append(st["colors_used"])
+    wm = float(np.mean(wms))
+    alg = GC_BYTES_PER_TASK * np.mean(pops) + GC_BYTES_PER_EDGE * np.mean(edges)
+    res["color"] = {"config": f"C4: Kronecker scale {args.gc_scale} ef 64 seed 4 (n={g.n}, m={g.m}), seed 1, warp worker",
+                    "ms_to_converge": float(np.mean(ms)), "ms_min": float(np.min(ms)), "worker_ms": wm,
+                    "colors": int(np.max(cols)), "tasks_per_n": float(np.mean(pops)) / g.n,
+                    "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak}
+    del csr, g, out
+    torch.cuda.empty_cache()
+    return res
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=8)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="atos", choices=["atos", "reference"])
+    ap.add_argument("--scale", type=int, default=26)
+    ap.add_argument("--pr-scale", type=int, default=22)
+    ap.add_argument("--gc-scale", type=int, default=20)
+    ap.add_argument("--app-steps", type=int, default=3)
+    ap.add_argument("--worker", type=int, default=256)
+    ap.add_argument("--fetch", type=int, default=256)
+    ap.add_argument("--no-apps", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        log("[bench] warmup raised to 3 (timing rules)")
+        args.warmup = 3
+    ws, rank, local = dist_setup()
+    if args.impl == "reference":
+        run_reference(args, ws, rank)
+    else:
+        run_atos(args, ws, rank, local)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -83,7 +83,9 @@ typedef struct {
     double   kernel_ms;         /* device time of the whole call (init + kernels + exchanges), CUDA events */
     double   residual_sum;      /* PageRank: sum of residues at exit (unnormalised), for conservation checks */
     int64_t  colors_used;       /* colouring: max colour + 1 */
-    uint64_t reserved[4];
+    double   worker_ms;         /* device time of the worker kernel(s) alone (persistent launch, or the sum
+                                   of the discrete launches incl. their host round trips), CUDA events */
+    uint64_t reserved[3];
 } atos_stats;
 
 typedef struct {

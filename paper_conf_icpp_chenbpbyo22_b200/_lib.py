@@ -35,7 +35,8 @@ class Stats(ctypes.Structure):
     _fields_ = [
         ("pops", ctypes.c_uint64), ("pushes", ctypes.c_uint64), ("edges", ctypes.c_uint64),
         ("rounds", ctypes.c_uint64), ("bytes_exchanged", ctypes.c_uint64), ("kernel_ms", ctypes.c_double),
-        ("residual_sum", ctypes.c_double), ("colors_used", ctypes.c_int64), ("reserved", ctypes.c_uint64 * 4),
+        ("residual_sum", ctypes.c_double), ("colors_used", ctypes.c_int64), ("worker_ms", ctypes.c_double),
+        ("reserved", ctypes.c_uint64 * 3),
     ]
 
     def as_dict(self):

@@ -534,6 +534,8 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   P.h0 = P.t0 = 0;
   const int mode = mode_of(r.worker);
   int rc;
+  WorkerTimer wt;
+  wt.start(s);
   if (mode == MODE_WARP) {
     const int block = r.block_threads, nw = block / 32;
     const size_t smem = (size_t)nw * 64 * 4 + (size_t)nw * 32 * 4 + group_smem_bytes<uint32_t>(r.fetch) * nw;
@@ -550,7 +552,9 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
     rc = launch_color_kernel(k_color_thread<true>, k_color_thread<false>, c, P, r, block, smem,
                              (uint64_t)r.fetch * 32 * nw, p, st);
   }
+  wt.stop(s);
   if (rc != ATOS_OK) return rc;
+  if (st) st->worker_ms += wt.elapsed();
   rc = finish_queue(p, s, st, "color");
   if (rc != ATOS_OK) return rc;
   unsigned long long* mx = p.scratch.as<unsigned long long>();

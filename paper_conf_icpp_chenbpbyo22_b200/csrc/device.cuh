@@ -154,34 +154,70 @@ __device__ __forceinline__ unsigned long long splitmix64(unsigned long long x) {
 }
 
 // -------------------------------------------------------------------- pushing
-// Publish `item` at reserved index idx: wait (bounded) until the slot is free
-// for this lap, then one release store of (idx+1, item).
-__device__ __forceinline__ void publish_one(const Ring& q, unsigned long long idx, uint32_t item,
-                                            unsigned long long watchdog_ns) {
-  unsigned long long* slot = q.slots + (idx & q.mask);
-  if ((uint32_t)(ld_relaxed(slot) >> 32) != (uint32_t)idx) {
-    // the previous lap's item in this slot has not been consumed yet: wait, bounded
-    unsigned long long t0 = globaltimer();
-    while ((uint32_t)(ld_relaxed(slot) >> 32) != (uint32_t)idx) {
-      __nanosleep(256);
-      if (globaltimer() - t0 > watchdog_ns) {
-        atomicOr((unsigned int*)&q.ctl->status.v, kStatusOverflow);
-        return;
-      }
-    }
-  }
-  st_release(slot, make_slot(idx + 1, item));
+__device__ __forceinline__ unsigned long long atom_cas_acq_rel(unsigned long long* p, unsigned long long cmp,
+                                                           unsigned long long val) {
+  unsigned long long old;
+  asm volatile("atom.acq_rel.gpu.global.cas.b64 %0, [%1], %2, %3;"
+               : "=l"(old) : "l"(p), "l"(cmp), "l"(val) : "memory");
+  return old;
 }
 
-// Try to take the item of index idx: true + *item on success (slot freed for the next lap).
-__device__ __forceinline__ bool try_consume(const Ring& q, unsigned long long idx, uint32_t* item) {
+// Publish `item` at reserved index idx.  Normally the slot is free for this
+// lap (seq == idx) and one release store publishes (idx+1, item).  If the slot
+// still holds the previous lap's item (seq == idx-C+1) because its claimant is
+// busy, the producer STEALS it with one CAS that publishes its own item in the
+// same step, then re-publishes the stolen item at a freshly reserved index and
+// counts the stolen index as done (after the re-publication, so termination
+// can never be observed early).  The claimant sees the slot's seq past its
+// index and drops the claim.  Producers therefore never wait on a busy
+// consumer; they only wait (bounded, watchdog) for a previous-lap producer
+// that reserved but has not yet written.
+__device__ __forceinline__ void publish_one(const Ring& q, unsigned long long idx, uint32_t item,
+                                            unsigned long long watchdog_ns) {
+  const unsigned long long C = q.mask + 1;
+  unsigned long long stolen = 0, t0 = 0;
+  while (true) {
+    unsigned long long* slot = q.slots + (idx & q.mask);
+    const unsigned long long v = ld_relaxed(slot);
+    const uint32_t seq = (uint32_t)(v >> 32);
+    if (seq == (uint32_t)idx) {
+      st_release(slot, make_slot(idx + 1, item));
+      break;
+    }
+    if (seq == (uint32_t)(idx - C + 1)) {
+      // previous lap's item still unconsumed: swap ours in, take it along
+      if (atom_cas_acq_rel(slot, v, make_slot(idx + 1, item)) == v) {
+        item = (uint32_t)v;
+        ++stolen;
+        idx = atomicAdd(&q.ctl->tail.v, 1ull);
+        t0 = 0;
+      }
+      continue;
+    }
+    // the previous lap's producer has reserved but not yet written: wait, bounded
+    if (t0 == 0) t0 = globaltimer();
+    else if (globaltimer() - t0 > watchdog_ns) {
+      atomicOr((unsigned int*)&q.ctl->status.v, kStatusOverflow);
+      break;
+    }
+    __nanosleep(64);
+  }
+  if (stolen) atom_add_release(&q.ctl->done.v, stolen);
+}
+
+// Try to take the item of index idx: 1 = taken (*item set, slot freed for the
+// next lap), 0 = not published yet, -1 = the item was stolen by a lap-blocked
+// producer (drop the claim).
+__device__ __forceinline__ int try_consume(const Ring& q, unsigned long long idx, uint32_t* item) {
   unsigned long long* slot = q.slots + (idx & q.mask);
   unsigned long long v;
   asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(slot) : "memory");
-  if ((uint32_t)(v >> 32) != (uint32_t)(idx + 1)) return false;
+  const int32_t d = (int32_t)((uint32_t)(v >> 32) - (uint32_t)(idx + 1));
+  if (d < 0) return 0;
+  if (d > 0) return -1;
+  if (atom_cas_acq_rel(slot, v, make_slot(idx + q.mask + 1, 0u)) != v) return -1;
   *item = (uint32_t)v;
-  st_relaxed(slot, make_slot(idx + q.mask + 1, 0u));
-  return true;
+  return 1;
 }
 
 // Per-warp staging buffer in shared memory.  push() is warp-collective (all 32

@@ -96,10 +96,11 @@ template <class Payload>
 __device__ __forceinline__ void consume_slot(const Ring& q, const GroupSmem<Payload>& s,
                                              unsigned long long idx) {
   uint32_t v;
-  if (!try_consume(q, idx, &v)) {
+  const int rc = try_consume(q, idx, &v);
+  if (rc == 0) {
     uint32_t k = atomicAdd(&s.ctr[2], 1u);
     s.pend2[k] = idx;
-  } else {
+  } else if (rc > 0) {
     uint32_t k = atomicAdd(&s.ctr[0], 1u);
     s.item[k] = v;
   }

@@ -134,6 +134,25 @@ struct CallTimer {
   }
 };
 
+// events around the worker kernel(s) of one call; elapsed() after the stream synchronised
+struct WorkerTimer {
+  cudaEvent_t a = nullptr, b = nullptr;
+  void start(cudaStream_t s) {
+    if (!a) { cudaEventCreate(&a); cudaEventCreate(&b); }
+    cudaEventRecord(a, s);
+  }
+  void stop(cudaStream_t s) { cudaEventRecord(b, s); }
+  double elapsed() {
+    float ms = 0;
+    if (a && cudaEventSynchronize(b) == cudaSuccess) cudaEventElapsedTime(&ms, a, b);
+    return ms;
+  }
+  ~WorkerTimer() {
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+  }
+};
+
 // wait for the stream, honouring cfg.timeout_s (polling) -- returns ATOS_ERR_TIMEOUT on expiry
 int stream_wait(cudaStream_t s, double timeout_s);
 

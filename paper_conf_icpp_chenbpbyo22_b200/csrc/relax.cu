@@ -23,9 +23,11 @@ __device__ __forceinline__ void run_begin(QueueCtl* ctl) {
 }
 
 // Before every persistent launch: over-claims abandoned by a previous kernel
-// of the same run are dropped (nothing is in flight between launches).
+// of the same run are dropped.  Between launches nothing is in flight and the
+// previous kernel consumed everything below `done`, so the unconsumed items
+// are exactly [done, tail).
 __global__ void k_sync_head(QueueCtl* ctl) {
-  if (threadIdx.x == 0 && blockIdx.x == 0) ctl->head.v = ctl->tail.v;
+  if (threadIdx.x == 0 && blockIdx.x == 0) ctl->head.v = ctl->done.v;
 }
 
 __global__ void k_run_begin(QueueCtl* ctl) {
@@ -211,7 +213,20 @@ static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, 
 }
 
 template <class App>
+static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, Part& p, atos_stats* st);
+
+template <class App>
 static int launch_relax(const App& app, const Ring& q, const Resolved& r, Part& p, atos_stats* st) {
+  WorkerTimer wt;
+  wt.start(r.stream);
+  const int rc = launch_relax_inner(app, q, r, p, st);
+  wt.stop(r.stream);
+  if (rc == ATOS_OK && st) st->worker_ms += wt.elapsed();
+  return rc;
+}
+
+template <class App>
+static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, Part& p, atos_stats* st) {
   EngineParams P;
   P.q = q;
   P.fetch = (uint32_t)r.fetch;
