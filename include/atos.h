@@ -85,7 +85,8 @@ typedef struct {
     int64_t  colors_used;       /* colouring: max colour + 1 */
     double   worker_ms;         /* device time of the worker kernel(s) alone (persistent launch, or the sum
                                    of the discrete launches incl. their host round trips), CUDA events */
-    uint64_t reserved[3];
+    uint64_t timeline_len;      /* samples written to cfg->timeline */
+    uint64_t reserved[2];
 } atos_stats;
 
 typedef struct {
@@ -109,7 +110,16 @@ typedef struct {
     void*    stream;            /* cudaStream_t; NULL = legacy default stream */
     atos_stats* stats;          /* optional out */
     int      l2_persist;        /* 1: L2 persisting access-policy window on queue counters + hot state */
-    int      reserved_i[7];
+    int      big_threshold;     /* persistent CTA/warp workers: a popped vertex with more edges than this is
+                                   split into chunks any worker may claim (hub assist); 0 = auto, <0 = off */
+    int      big_chunk;         /* edges per hub-assist chunk; 0 = auto */
+    uint32_t timeline_cap;      /* samples available in `timeline` (0 = no timeline) */
+    uint64_t* timeline;         /* optional DEVICE buffer of 4*timeline_cap uint64: progress samples
+                                   (globaltimer ns, tasks done, queue tail, queue head) taken by the
+                                   workers every timeline_interval_ns -- the throughput-vs-time data of
+                                   the paper's Figs. 1-3 */
+    uint32_t timeline_interval_ns; /* 0 = 5000 */
+    int      reserved_i[3];
 } atos_cfg;
 
 /* Fill *cfg with defaults (persistent, app-default worker/fetch, dedupe on). */

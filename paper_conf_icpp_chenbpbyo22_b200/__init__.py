@@ -75,7 +75,13 @@ class CSR:
 def _run(fn_name: str, g: CSR, out: torch.Tensor, args: tuple, stream, knobs: dict):
     lib = _lib.load()
     st = Stats()
+    timeline = knobs.pop("timeline", None)
     cfg = default_cfg(**knobs)
+    if timeline is not None:
+        if not (timeline.is_cuda and timeline.dtype == torch.int64 and timeline.is_contiguous()):
+            raise TypeError("timeline must be a contiguous int64 CUDA tensor of 4*cap entries")
+        cfg.timeline = ctypes.c_void_p(timeline.data_ptr())
+        cfg.timeline_cap = timeline.numel() // 4
     cfg.stats = ctypes.pointer(st)
     if out.is_cuda:
         cfg.out_where = _lib.MEM_DEVICE
@@ -113,6 +119,16 @@ def color(g: CSR, seed: int = 1, out: torch.Tensor | None = None, stream=None, *
     if out is None:
         out = torch.empty(g.n, dtype=torch.int32, device=f"cuda:{g.device}")
     return _run("atos_color", g, out, (ctypes.c_uint64(seed & (2**64 - 1)),), stream, knobs)
+
+
+def timeline_table(timeline: torch.Tensor, stats: dict):
+    """Samples (t_us from the first sample, done, tail, head) of a cfg.timeline buffer."""
+    k = min(int(stats.get("timeline_len", 0)), timeline.numel() // 4)
+    t = timeline[: 4 * k].view(k, 4).cpu()
+    if k:
+        t = t.clone()
+        t[:, 0] -= t[0, 0].item()
+    return t
 
 
 def launches() -> int:

@@ -36,7 +36,7 @@ class Stats(ctypes.Structure):
         ("pops", ctypes.c_uint64), ("pushes", ctypes.c_uint64), ("edges", ctypes.c_uint64),
         ("rounds", ctypes.c_uint64), ("bytes_exchanged", ctypes.c_uint64), ("kernel_ms", ctypes.c_double),
         ("residual_sum", ctypes.c_double), ("colors_used", ctypes.c_int64), ("worker_ms", ctypes.c_double),
-        ("reserved", ctypes.c_uint64 * 3),
+        ("timeline_len", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 2),
     ]
 
     def as_dict(self):
@@ -50,7 +50,9 @@ class Cfg(ctypes.Structure):
         ("dedupe", ctypes.c_int), ("check_size", ctypes.c_int), ("conflict_policy", ctypes.c_int),
         ("permute_init", ctypes.c_int), ("validate", ctypes.c_int), ("out_where", ctypes.c_int),
         ("queue_capacity", ctypes.c_uint64), ("timeout_s", ctypes.c_double), ("stream", ctypes.c_void_p),
-        ("stats", ctypes.POINTER(Stats)), ("l2_persist", ctypes.c_int), ("reserved_i", ctypes.c_int * 7),
+        ("stats", ctypes.POINTER(Stats)), ("l2_persist", ctypes.c_int), ("big_threshold", ctypes.c_int),
+        ("big_chunk", ctypes.c_int), ("timeline_cap", ctypes.c_uint32), ("timeline", ctypes.c_void_p),
+        ("timeline_interval_ns", ctypes.c_uint32), ("reserved_i", ctypes.c_int * 3),
     ]
 
 

@@ -88,6 +88,15 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
     return ATOS_ERR_INVALID_ARG;
   }
   r->l2_persist = d.l2_persist;
+  r->timeline = (unsigned long long*)d.timeline;
+  r->timeline_cap = d.timeline ? d.timeline_cap : 0;
+  r->timeline_interval_ns = d.timeline_interval_ns ? d.timeline_interval_ns : 5000;
+  r->big_threshold = d.big_threshold;
+  r->big_chunk = d.big_chunk;
+  if (r->big_chunk < 0) {
+    set_error("big_chunk must be >= 0");
+    return ATOS_ERR_INVALID_ARG;
+  }
   r->queue_capacity = d.queue_capacity;
   r->timeout_s = d.timeout_s;
   if (r->timeout_s < 0) {
@@ -101,15 +110,25 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
 }
 
 // Fresh ring: slot i free for index i (seq = i), all counters 0.
-__global__ void k_ring_init(unsigned long long* slots, unsigned long long cap, QueueCtl* ctl) {
+__global__ void k_ring_init(unsigned long long* slots, unsigned long long cap, QueueCtl* ctl, BigTask* big,
+                            uint32_t nbig) {
   for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < cap;
        i += (unsigned long long)gridDim.x * blockDim.x)
     slots[i] = make_slot(i, 0u);
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    ctl->head.v = 0;
-    ctl->tail.v = 0;
-    ctl->done.v = 0;
-    ctl->status.v = 0;
+  if (blockIdx.x == 0) {
+    for (uint32_t i = threadIdx.x; i < nbig; i += blockDim.x) {
+      big[i].state = 0;
+      big[i].gen = 0;
+      big[i].ctr = 0;
+    }
+    if (threadIdx.x == 0) {
+      ctl->head.v = 0;
+      ctl->tail.v = 0;
+      ctl->done.v = 0;
+      ctl->status.v = 0;
+      ctl->big_count.v = 0;
+      ctl->big_rr.v = 0;
+    }
   }
 }
 
@@ -120,9 +139,11 @@ int ensure_queue(Part& p, uint64_t cap, cudaStream_t s) {
     p.ring_clean = false;
   }
   if (!p.ctl.p) ATOS_TRY(p.ctl.ensure(sizeof(QueueCtl)));
+  if (!p.big.p) ATOS_TRY(p.big.ensure(sizeof(BigTask) * kBigSlots));
   if (!p.host_pinned) ATOS_CUDA(cudaHostAlloc(&p.host_pinned, 4096, cudaHostAllocDefault));
   if (!p.ring_clean) {
-    k_ring_init<<<1184, 256, 0, s>>>(p.ring.as<unsigned long long>(), p.ring_cap, p.ctl.as<QueueCtl>());
+    k_ring_init<<<1184, 256, 0, s>>>(p.ring.as<unsigned long long>(), p.ring_cap, p.ctl.as<QueueCtl>(),
+                                     p.big.as<BigTask>(), kBigSlots);
     g_launches++;
     ATOS_CUDA(cudaGetLastError());
     p.ring_clean = true;
@@ -214,6 +235,7 @@ int finish_queue(Part& p, cudaStream_t s, atos_stats* st, const char* what) {
     st->pops += h->stat_pops.v;
     st->pushes += h->stat_pushes.v;
     st->edges += h->stat_edges.v;
+    st->timeline_len = h->tl_count.v;
   }
   return ATOS_OK;
 }
@@ -326,7 +348,7 @@ void destroy_part(Part& p) {
   if (p.col) cudaFree(p.col);
   p.row_ptr = nullptr;
   p.col = nullptr;
-  DevBuf* bufs[] = {&p.ring, &p.ctl, &p.bitmap, &p.vbuf_a, &p.vbuf_b, &p.vbuf_c, &p.scratch,
+  DevBuf* bufs[] = {&p.ring, &p.ctl, &p.big, &p.bitmap, &p.shadow, &p.vbuf_a, &p.vbuf_b, &p.vbuf_c, &p.scratch,
                     &p.ghost_a, &p.ghost_b, &p.touched, &p.outbox, &p.inbox};
   for (DevBuf* b : bufs) b->release();
   if (p.host_pinned) cudaFreeHost(p.host_pinned);

@@ -15,12 +15,26 @@ namespace atos {
 //     release RMW after its atomicMin and pushes only if the bit was clear;
 //     the popper clears it with an acquire RMW BEFORE reading depth[v], so
 //     every improvement after that read re-queues v (no update is lost).
+//   * shadow depth (B200 addition): a u8 copy
+//     min(depth, 254) with 255 = "unvisited or >= 255", n bytes (67 MB at
+//     scale 26) -- small enough to stay in the 126 MB L2 (loads evict_last,
+//     the col stream evict_first), so the per-edge prefilter almost never
+//     touches HBM.  Written after a successful atomicMin; concurrent writers
+//     can only leave a value depth[w] once held, so it stays an upper bound.
 struct BfsApp {
   using Payload = uint32_t;  // d + 1
   const uint32_t* __restrict__ row_ptr;
   const uint32_t* __restrict__ col;
   uint32_t* depth;
-  uint32_t* inq;  // nullptr -> paper-literal push on every improvement
+  uint32_t* inq;      // nullptr -> paper-literal push on every improvement
+  uint8_t* shadow;    // nullptr -> prefilter on depth[] itself
+  unsigned long long pol_first, pol_last;
+
+  __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
+  __device__ __forceinline__ void prepare() {
+    pol_first = policy_evict_first();
+    pol_last = policy_evict_last();
+  }
 
   __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
     if (inq) atom_and_acquire(inq + (v >> 5), ~(1u << (v & 31)));
@@ -32,11 +46,20 @@ struct BfsApp {
   }
 
   __device__ __forceinline__ bool relax(const Payload nd, uint32_t w, uint32_t& out) const {
-    uint32_t cur;
-    asm volatile("ld.global.u32 %0, [%1];" : "=r"(cur) : "l"(depth + w));
-    if (cur <= nd) return false;
+    bool need_depth_check = true;
+    if (shadow) {
+      const uint32_t sh = ld_u8_hint(shadow + w, pol_last);
+      if (sh != 255u && sh <= nd) return false;
+      need_depth_check = nd >= 255u;  // sh == 255 && nd < 255: unvisited or deeper -> must improve
+    }
+    if (need_depth_check) {
+      uint32_t cur;
+      asm volatile("ld.global.u32 %0, [%1];" : "=r"(cur) : "l"(depth + w));
+      if (cur <= nd) return false;
+    }
     const uint32_t old = atomicMin(depth + w, nd);
     if (old <= nd) return false;
+    if (shadow) st_u8_hint(shadow + w, nd < 255u ? nd : 255u, pol_last);
     if (inq) {
       const uint32_t bit = 1u << (w & 31);
       if (atom_or_release(inq + (w >> 5), bit) & bit) return false;
@@ -57,6 +80,9 @@ struct PrApp {
   using Payload = double;  // delta = alpha * rho / deg(v)
   const uint32_t* __restrict__ row_ptr;
   const uint32_t* __restrict__ col;
+  unsigned long long pol_first;
+  __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
+  __device__ __forceinline__ void prepare() { pol_first = policy_evict_first(); }
   double* rank;
   double* res;
   double alpha, eps;

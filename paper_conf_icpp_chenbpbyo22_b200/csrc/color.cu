@@ -396,6 +396,8 @@ __global__ void k_color_begin(QueueCtl* ctl, unsigned long long n) {
     ctl->stat_pushes.v = n;
     ctl->stat_edges.v = 0;
     ctl->misc.v = 0;
+    ctl->tl_next.v = 0;
+    ctl->tl_count.v = 0;
   }
 }
 
@@ -532,6 +534,13 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   P.fetch = (uint32_t)r.fetch;
   P.watchdog_ns = r.watchdog_ns;
   P.h0 = P.t0 = 0;
+  P.tl = r.timeline;
+  P.tl_cap = r.timeline_cap;
+  P.tl_interval_ns = r.timeline_interval_ns;
+  P.big = nullptr;
+  P.nbig = 0;
+  P.big_threshold = 0xFFFFFFFFu;
+  P.big_chunk = 1;
   const int mode = mode_of(r.worker);
   int rc;
   WorkerTimer wt;

@@ -51,6 +51,10 @@ struct QueueCtl {
   Line64 stat_pushes;
   Line64 stat_edges;
   Line64 misc;        // app scratch (e.g. colouring: max colour)
+  Line64 big_count;   // active big tasks (hub assist)
+  Line64 big_rr;      // round-robin slot cursor for big-task registration
+  Line64 tl_next;     // timeline: globaltimer of the next sample
+  Line64 tl_count;    // timeline: samples taken
 };
 
 struct Ring {
@@ -133,6 +137,33 @@ __device__ __forceinline__ unsigned long long atom_read(unsigned long long* p) {
 __device__ __forceinline__ void red_add_f64(double* p, double v) {
   asm volatile("red.relaxed.gpu.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
 }
+// L2 eviction-priority policies (createpolicy) and hinted loads: graph
+// streams (col) are evict_first so they do not push the small hot state
+// (shadow depth, bitmaps) out of the 126 MB L2.
+__device__ __forceinline__ unsigned long long policy_evict_first() {
+  unsigned long long p;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ unsigned long long policy_evict_last() {
+  unsigned long long p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint32_t ld_stream(const uint32_t* a, unsigned long long pol) {
+  uint32_t v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(a), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_u8_hint(const uint8_t* a, unsigned long long pol) {
+  uint16_t v;
+  asm volatile("ld.global.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(a), "l"(pol) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_u8_hint(uint8_t* a, uint32_t v, unsigned long long pol) {
+  asm volatile("st.global.L2::cache_hint.u8 [%0], %1, %2;" ::"l"(a), "h"((uint16_t)v), "l"(pol) : "memory");
+}
+
 __device__ __forceinline__ void fence_sc_gpu() { asm volatile("fence.sc.gpu;" ::: "memory"); }
 __device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 

@@ -34,12 +34,160 @@ namespace atos {
 
 enum { MODE_CTA = 0, MODE_WARP = 1, MODE_THREAD = 2 };
 
+// ------------------------------------------------------------ big-task assist
+// A popped vertex whose degree exceeds big_threshold is not expanded by the
+// worker that popped it: it is registered in a small global table and its
+// edge list is split into big_chunk-edge chunks that ANY worker claims with
+// one atomicAdd -- busy workers check the table before fetching new items and
+// idle workers are sent there first.  This extends the paper's CTA-internal
+// data-parallel balancing across CTAs for hubs, which otherwise
+// pin one worker for milliseconds on scale-free graphs.  The
+// popped item counts as done only when its last chunk finishes, so the
+// queue's termination rule is unchanged.  (DESIGN.md "Big-task assist".)
+struct __align__(64) BigTask {
+  unsigned long long ctr;      // (generation << 32) | next chunk
+  unsigned long long payload;  // Payload bits
+  uint32_t state;              // 0 free, 1 filling, 2 active
+  uint32_t gen;
+  uint32_t v, start, deg, nchunks, finished, pad;
+  unsigned long long pad2[2];
+};
+
 struct EngineParams {
   Ring q;
   uint32_t fetch;                   // items per claim per worker (per lane for THREAD)
   unsigned long long watchdog_ns;   // spin budget before the watchdog trips
   unsigned long long h0, t0;        // discrete mode: the frontier [h0, t0)
+  BigTask* big;                     // nullptr: no assist
+  uint32_t nbig, big_threshold, big_chunk;
+  unsigned long long* tl;           // progress timeline (nullptr: off)
+  uint32_t tl_cap, tl_interval_ns;
 };
+
+// Progress sample (globaltimer, done, tail, head) at most every tl_interval_ns,
+// taken by whichever worker first notices the sampling time has passed.
+__device__ __forceinline__ void tl_sample(const EngineParams& P) {
+  if (!P.tl) return;
+  QueueCtl* c = P.q.ctl;
+  const unsigned long long now = globaltimer();
+  const unsigned long long nxt = ld_relaxed(&c->tl_next.v);
+  if (now < nxt) return;
+  if (atomicCAS(&c->tl_next.v, nxt, now + P.tl_interval_ns) != nxt) return;
+  const unsigned long long k = atomicAdd(&c->tl_count.v, 1ull);
+  if (k >= P.tl_cap) return;
+  unsigned long long* e = P.tl + 4 * k;
+  e[0] = now;
+  e[1] = ld_relaxed(&c->done.v);
+  e[2] = ld_relaxed(&c->tail.v);
+  e[3] = ld_relaxed(&c->head.v);
+}
+
+constexpr uint32_t kGoBig = 0xFFFFFFFFu;
+
+template <class Payload>
+__device__ __forceinline__ unsigned long long payload_bits(const Payload& p) {
+  static_assert(sizeof(Payload) <= 8, "payload must fit 8 bytes");
+  unsigned long long b = 0;
+  memcpy(&b, &p, sizeof(Payload));
+  return b;
+}
+template <class Payload>
+__device__ __forceinline__ Payload payload_from(unsigned long long b) {
+  Payload p;
+  memcpy(&p, &b, sizeof(Payload));
+  return p;
+}
+
+// Register item v (row [start, start+deg), payload p) as a big task.  False
+// when no free slot was found (the caller expands the vertex itself).
+// Order: state 0->1 (CAS) ; fields ; gen+1 (atomic) ; ctr = gen<<32 ; state = 2.
+template <class Payload>
+__device__ __forceinline__ bool register_big(const EngineParams& P, uint32_t v, uint32_t start, uint32_t deg,
+                                             const Payload& p) {
+  const uint32_t slot = (uint32_t)(atomicAdd(&P.q.ctl->big_rr.v, 1ull) % P.nbig);
+  BigTask* t = P.big + slot;
+  if (atomicCAS(&t->state, 0u, 1u) != 0u) return false;
+  t->v = v;
+  t->start = start;
+  t->deg = deg;
+  t->nchunks = (deg + P.big_chunk - 1) / P.big_chunk;
+  t->finished = 0;
+  t->payload = payload_bits(p);
+  const uint32_t gen = atomicAdd(&t->gen, 1u) + 1u;  // RMW: monotone, never a stale read
+  __threadfence();
+  atomicExch(&t->ctr, (unsigned long long)gen << 32);
+  __threadfence();
+  atomicExch(&t->state, 2u);
+  atomicAdd(&P.q.ctl->big_count.v, 1ull);
+  return true;
+}
+
+// Warp-collective: claim one chunk of an active big task.  Returns the slot
+// (or -1) and sets chunk; every lane gets the same answer.  When a chunk is
+// claimed, lane 0 (which performed the acquire) writes the task fields to
+// out[0..3] = start, deg, payload lo, payload hi (shared memory).
+// A counter increment is valid only if, once the slot is active again, the
+// slot's generation still equals the one carried by the counter value and the
+// chunk index is in range -- so late claims on a retired/reused slot are
+// rejected and no chunk is ever processed twice.
+__device__ __forceinline__ int claim_big_warp(const EngineParams& P, uint32_t& chunk, uint32_t* out) {
+  if (ld_relaxed(&P.q.ctl->big_count.v) == 0) return -1;
+  for (uint32_t base = 0; base < P.nbig; base += 32) {
+    const uint32_t i = base + lane_id();
+    bool act = false;
+    if (i < P.nbig) {
+      const BigTask* t = P.big + i;
+      act = ld_relaxed(&t->state) == 2u && (uint32_t)ld_relaxed(&t->ctr) < ld_relaxed(&t->nchunks);
+    }
+    unsigned m = __ballot_sync(0xffffffffu, act);
+    while (m) {
+      const uint32_t L = __ffs(m) - 1;
+      m &= m - 1;
+      BigTask* t = P.big + base + L;
+      int ok = 0;
+      uint32_t c = 0;
+      if (lane_id() == 0) {
+        const unsigned long long old = atomicAdd(&t->ctr, 1ull);
+        const uint32_t gen = (uint32_t)(old >> 32);
+        c = (uint32_t)old;
+        uint32_t st = ld_acquire(&t->state);
+        while (st == 1u) {  // a registration is filling the slot: wait for it to settle
+          __nanosleep(32);
+          st = ld_acquire(&t->state);
+        }
+        if (st == 2u && ld_relaxed(&t->gen) == gen && c < ld_relaxed(&t->nchunks)) {
+          ok = 1;
+          out[0] = ld_relaxed(&t->start);
+          out[1] = ld_relaxed(&t->deg);
+          const unsigned long long pb = ld_relaxed(&t->payload);
+          out[2] = (uint32_t)pb;
+          out[3] = (uint32_t)(pb >> 32);
+        }
+      }
+      ok = __shfl_sync(0xffffffffu, ok, 0);
+      c = __shfl_sync(0xffffffffu, c, 0);
+      if (ok) {
+        chunk = c;
+        return (int)(base + L);
+      }
+    }
+  }
+  return -1;
+}
+
+// A chunk is finished (its pushes published): the last finisher retires the
+// task and counts the original item as done.
+__device__ __forceinline__ void finish_big_chunk(const EngineParams& P, int slot) {
+  BigTask* t = P.big + slot;
+  fence_acq_rel_gpu();
+  const uint32_t f = atomicAdd(&t->finished, 1u);
+  if (f + 1 == ld_relaxed(&t->nchunks)) {
+    fence_acq_rel_gpu();
+    atomicExch(&t->state, 0u);
+    atomicAdd(&P.q.ctl->big_count.v, (unsigned long long)-1ll);
+    atom_add_release(&P.q.ctl->done.v, 1ull);
+  }
+}
 
 // Per-group shared-memory arena.  K = items a group may hold at once.
 template <class Payload>
@@ -142,7 +290,7 @@ struct Worker {
     while (true) {
       // ------------------------------------------------------ 1. claim
       if (r == 0) {
-        s.ctr[0] = 0; s.ctr[2] = 0; s.ctr[3] = 0; s.ctr[4] = 0;
+        s.ctr[0] = 0; s.ctr[2] = 0; s.ctr[3] = 0; s.ctr[4] = 0; s.ctr[5] = 0;
         *(unsigned long long*)&s.ctr[6] = 0;
         if (!PERSIST) {
           if (!first) {
@@ -195,6 +343,9 @@ struct Worker {
         const uint32_t st = *(volatile uint32_t*)&q.ctl->status.v;
         if (d == t || st != 0) {
           s.ctr[3] = 1;
+        } else if (PERSIST && P.nbig && ld_relaxed(&q.ctl->big_count.v) != 0) {
+          tl_sample(P);
+          s.ctr[3] = 2;  // go help with big tasks
         } else {
           const unsigned long long now = globaltimer();
           if (idle_since == 0) idle_since = now;
@@ -202,11 +353,13 @@ struct Worker {
             atomicOr((unsigned int*)&q.ctl->status.v, kStatusTimeout);
             s.ctr[3] = 1;
           }
+          tl_sample(P);
           __nanosleep(backoff);
           backoff = backoff < 2048 ? backoff * 2 : 2048;
         }
       }
       group_sync<MODE>();
+      if (s.ctr[3] == 2) return kGoBig;
       if (s.ctr[3]) return 0;
     }
   }
@@ -215,10 +368,11 @@ struct Worker {
   // count the batch as done with release semantics.
   __device__ __forceinline__ void complete(const EngineParams& P, uint32_t nready) {
     group_sync<MODE>();
-    if (PERSIST && r == 0) {
+    if (PERSIST && r == 0 && nready) {
       fence_acq_rel_gpu();
       atom_add_release(&P.q.ctl->done.v, (unsigned long long)nready);
     }
+    if (r == 0) tl_sample(P);
     group_sync<MODE>();
   }
 };
@@ -251,21 +405,68 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
   WarpPusher pusher{pushbuf + warp_id() * 64, 0, 0};
   unsigned long long my_pops = 0, my_edges = 0;
   const Ring& q = P.q;
+  app.prepare();
+  constexpr bool kAssist = PERSIST && MODE != MODE_THREAD;
+  const bool assist = kAssist && P.nbig != 0;
 
   while (true) {
+    // ---------------------------------------------------------- 0. big-task chunks first
+    if (assist) {
+      if (MODE == MODE_CTA) {
+        if (warp_id() == 0) {
+          uint32_t c = 0;
+          const int slot = claim_big_warp(P, c, s.ctr + 43);
+          if (lane_id() == 0) { s.ctr[41] = (uint32_t)slot; s.ctr[42] = c; }
+        }
+        __syncthreads();
+      } else {
+        uint32_t c = 0;
+        const int slot = claim_big_warp(P, c, s.ctr + 43);
+        if (lane_id() == 0) { s.ctr[41] = (uint32_t)slot; s.ctr[42] = c; }
+        __syncwarp();
+      }
+      const int slot = (int)s.ctr[41];
+      if (slot >= 0) {
+        const uint32_t c = s.ctr[42];
+        const uint32_t b0 = c * P.big_chunk;
+        const uint32_t len = min(P.big_chunk, s.ctr[44] - b0);
+        const uint32_t st0 = s.ctr[43] + b0;
+        const Payload p = payload_from<Payload>(((unsigned long long)s.ctr[46] << 32) | s.ctr[45]);
+        my_edges += (r == 0) ? len : 0;
+        for (uint32_t base = 0; base < len; base += G) {
+          const uint32_t e = base + r;
+          bool want = false;
+          uint32_t out = 0;
+          if (e < len) want = app.relax(p, app.neighbor(st0 + e), out);
+          pusher.push(q, want, out, P.watchdog_ns);
+        }
+        pusher.flush(q, P.watchdog_ns);
+        group_sync<MODE>();
+        if (r == 0) finish_big_chunk(P, slot);
+        group_sync<MODE>();
+        continue;
+      }
+      group_sync<MODE>();
+    }
     const uint32_t nready = wk.acquire(P);
+    if (nready == kGoBig) continue;
     if (nready == 0) break;
     // ---------------------------------------------------------- begin (per item)
     for (uint32_t k = r; k < nready; k += G) {
       uint32_t st = 0, dg = 0;
       Payload p{};
       if (!app.begin(s.item[k], st, dg, p)) dg = 0;
+      if (assist && dg > P.big_threshold && register_big(P, s.item[k], st, dg, p)) {
+        dg = 0;  // expanded by the assist chunks; counted done by the last chunk
+        atomicAdd(&s.ctr[5], 1u);
+      }
       s.start[k] = st;
       s.off[k] = dg;
       s.pay[k] = p;
     }
     group_sync<MODE>();
     my_pops += (r == 0) ? nready : 0;
+    const uint32_t deferred = s.ctr[5];
 
     // ---------------------------------------------------------- expand + relax
     if (MODE == MODE_CTA) {
@@ -290,7 +491,7 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
             const uint32_t mid = (lo + hi) >> 1;
             if (s.off[mid] <= e) lo = mid; else hi = mid;
           }
-          const uint32_t w = __ldg(app.col + s.start[lo] + (e - s.off[lo]));
+          const uint32_t w = app.neighbor(s.start[lo] + (e - s.off[lo]));
           want = app.relax(s.pay[lo], w, out);
         }
         pusher.push(q, want, out, P.watchdog_ns);
@@ -304,7 +505,7 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
           bool want = false;
           uint32_t out = 0;
           if (j + r < dg) {
-            const uint32_t w = __ldg(app.col + st + j + r);
+            const uint32_t w = app.neighbor(st + j + r);
             want = app.relax(p, w, out);
           }
           pusher.push(q, want, out, P.watchdog_ns);
@@ -326,7 +527,7 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
         bool want = false;
         uint32_t out = 0;
         if (active) {
-          const uint32_t w = __ldg(app.col + st + j);
+          const uint32_t w = app.neighbor(st + j);
           ++j;
           ++my_edges;
           want = app.relax(p, w, out);
@@ -335,7 +536,7 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
       }
     }
     pusher.flush(q, P.watchdog_ns);
-    wk.complete(P, nready);
+    wk.complete(P, nready - deferred);
   }
   flush_stats(q, my_pops, my_edges, lane_id() == 0 ? pusher.total : 0);
 }

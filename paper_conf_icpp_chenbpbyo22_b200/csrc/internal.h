@@ -50,7 +50,7 @@ struct Part {
   uint32_t* row_ptr = nullptr;      // n_local + 1, local offsets
   uint32_t* col = nullptr;          // m_local, GLOBAL ids (single-partition: the ids)
   // cached workspaces (grow-only, reused across calls)
-  DevBuf ring, ctl, bitmap, vbuf_a, vbuf_b, vbuf_c, scratch;
+  DevBuf ring, ctl, big, bitmap, shadow, vbuf_a, vbuf_b, vbuf_c, scratch;
   DevBuf ghost_a, ghost_b, touched, outbox, inbox;
   uint64_t ring_cap = 0;
   void* host_pinned = nullptr;      // 4 KB pinned scratch for control-block reads
@@ -91,7 +91,9 @@ struct DeviceGuard {
 
 struct Resolved {
   int persistent, worker, fetch, num_blocks, block_threads, dedupe, check_size;
-  int conflict_policy, permute_init, validate, out_where, l2_persist;
+  int conflict_policy, permute_init, validate, out_where, l2_persist, big_threshold, big_chunk;
+  unsigned long long* timeline;
+  uint32_t timeline_cap, timeline_interval_ns;
   uint64_t queue_capacity;
   double timeout_s;
   cudaStream_t stream;
@@ -105,7 +107,9 @@ inline int mode_of(int worker) {
   return worker == 1 ? MODE_THREAD : (worker == 32 ? MODE_WARP : MODE_CTA);
 }
 
-// Ring/control workspace of a partition: capacity >= want (power of two), all slots EMPTY.
+constexpr uint32_t kBigSlots = 64;
+
+// Ring/control workspace of a partition (+ the big-task table): capacity >= want (power of two), all slots EMPTY.
 int ensure_queue(Part& p, uint64_t want_cap, cudaStream_t s);
 // persistent grid size: occupancy max x SMs
 int persistent_grid(const void* fn, int block, size_t smem, int* grid);

@@ -20,6 +20,8 @@ __device__ __forceinline__ void run_begin(QueueCtl* ctl) {
   ctl->stat_pushes.v = 0;
   ctl->stat_edges.v = 0;
   ctl->misc.v = 0;
+  ctl->tl_next.v = 0;
+  ctl->tl_count.v = 0;
 }
 
 // Before every persistent launch: over-claims abandoned by a previous kernel
@@ -36,10 +38,12 @@ __global__ void k_run_begin(QueueCtl* ctl) {
 
 // BFS init (Alg.1 P:721-725 "vertex.dist = MAX_UINT32", frontier = [source];
 // source depth 0, R-BFS-1).  depth[] was memset to 0xFF on the stream.
-__global__ void k_bfs_init(uint32_t* depth, uint32_t* inq, Ring q, uint32_t src, unsigned long long wd) {
+__global__ void k_bfs_init(uint32_t* depth, uint32_t* inq, uint8_t* shadow, Ring q, uint32_t src,
+                           unsigned long long wd) {
   if (threadIdx.x == 0 && blockIdx.x == 0) {
     run_begin(q.ctl);
     depth[src] = 0;
+    if (shadow) shadow[src] = 0;
     if (inq) inq[src >> 5] |= 1u << (src & 31);
     const unsigned long long idx = q.ctl->tail.v;
     q.ctl->tail.v = idx + 1;
@@ -234,6 +238,22 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
   P.h0 = P.t0 = 0;
   const int mode = mode_of(r.worker);
   const int block = mode == MODE_CTA ? r.worker : r.block_threads;
+  // hub assist (persistent CTA / warp workers): auto threshold = 32 edges per
+  // worker thread, chunks of 8 edges per worker thread (>= 1024)
+  P.tl = r.timeline;
+  P.tl_cap = r.timeline_cap;
+  P.tl_interval_ns = r.timeline_interval_ns;
+  P.big = nullptr;
+  P.nbig = 0;
+  P.big_threshold = 0xFFFFFFFFu;
+  P.big_chunk = 1;
+  if (r.persistent && mode != MODE_THREAD && r.big_threshold >= 0 && p.big.p) {
+    const uint32_t wsz = mode == MODE_CTA ? (uint32_t)r.worker : 32u;
+    P.big = p.big.as<BigTask>();
+    P.nbig = kBigSlots;
+    P.big_threshold = r.big_threshold > 0 ? (uint32_t)r.big_threshold : std::max(4096u, 32u * wsz);
+    P.big_chunk = r.big_chunk > 0 ? (uint32_t)r.big_chunk : std::max(1024u, 8u * wsz);
+  }
   if (mode == MODE_CTA) return launch_relax_mode<App, MODE_CTA>(app, P, r, block, p, st);
   if (mode == MODE_WARP) return launch_relax_mode<App, MODE_WARP>(app, P, r, block, p, st);
   return launch_relax_mode<App, MODE_THREAD>(app, P, r, block, p, st);
@@ -261,12 +281,15 @@ int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolve
     ATOS_CUDA(cudaMemsetAsync(inq, 0, ((size_t)n + 31) / 32 * 4, s));
   }
   ATOS_CUDA(cudaMemsetAsync(depth, 0xFF, (size_t)n * 4, s));
+  ATOS_TRY(p.shadow.ensure((size_t)n));
+  uint8_t* shadow = p.shadow.as<uint8_t>();
+  ATOS_CUDA(cudaMemsetAsync(shadow, 0xFF, (size_t)n, s));
   Ring q = ring_of(p);
-  k_bfs_init<<<1, 32, 0, s>>>(depth, inq, q, (uint32_t)src, r.watchdog_ns);
+  k_bfs_init<<<1, 32, 0, s>>>(depth, inq, shadow, q, (uint32_t)src, r.watchdog_ns);
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, depth, (size_t)n * 4, true);
-  BfsApp app{p.row_ptr, p.col, depth, inq};
+  BfsApp app{p.row_ptr, p.col, depth, inq, shadow, 0ull, 0ull};
   p.ring_clean = false;
   int rc = launch_relax(app, q, r, p, st);
   if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
@@ -300,7 +323,7 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, res, (size_t)n * 8, true);
-  PrApp app{p.row_ptr, p.col, rank, res, alpha, eps, r.check_size > 0 ? 0 : 1};
+  PrApp app{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, r.check_size > 0 ? 0 : 1};
   p.ring_clean = false;
   int rc = ATOS_OK;
   if (r.check_size <= 0) {

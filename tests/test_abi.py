@@ -44,7 +44,7 @@ def test_cfg_layout_and_defaults():
     cfg = _lib.default_cfg()
     assert cfg.struct_size == ctypes.sizeof(_lib.Cfg)
     assert cfg.persistent == 1 and cfg.dedupe == 1 and cfg.out_where == _lib.MEM_DEVICE
-    assert ctypes.sizeof(_lib.Stats) == 9 * 8 + 8 * 3
+    assert ctypes.sizeof(_lib.Stats) == 10 * 8 + 8 * 2
 
 
 def test_partition_range():

@@ -32,6 +32,11 @@ KNOBS = [
     dict(worker=1, fetch_size=2, persistent=0),
     dict(worker=256, fetch_size=256, persistent=1, dedupe=0),
     dict(worker=32, fetch_size=4, persistent=1, dedupe=0),
+    # hub assist (big tasks) stressed with tiny thresholds/chunks, and disabled
+    dict(worker=256, fetch_size=256, big_threshold=64, big_chunk=16),
+    dict(worker=32, fetch_size=8, big_threshold=32, big_chunk=8),
+    dict(worker=128, fetch_size=32, big_threshold=8, big_chunk=1, dedupe=0),
+    dict(worker=256, fetch_size=256, big_threshold=-1),
 ]
 
 

@@ -23,6 +23,9 @@ KNOBS = [
     dict(worker=256, fetch_size=256, persistent=0),
     dict(worker=32, fetch_size=4, persistent=0),
     dict(worker=256, fetch_size=256, check_size=1024),
+    dict(worker=256, fetch_size=256, big_threshold=64, big_chunk=16),
+    dict(worker=32, fetch_size=4, big_threshold=16, big_chunk=4),
+    dict(worker=256, fetch_size=256, big_threshold=-1),
 ]
 
 
