@@ -1,6 +1,7 @@
 // api.cu -- the C ABI (include/atos.h): handles, configuration, errors, and
 // the host-side plumbing shared by all solvers.
 #include <cstdarg>
+#include <cstdlib>
 #include <cstring>
 #include <chrono>
 #include <thread>
@@ -118,8 +119,8 @@ __global__ void k_ring_init(unsigned long long* slots, unsigned long long cap, Q
   if (blockIdx.x == 0) {
     for (uint32_t i = threadIdx.x; i < nbig; i += blockDim.x) {
       big[i].state = 0;
-      big[i].gen = 0;
       big[i].ctr = 0;
+      big[i].finished = 0;
     }
     if (threadIdx.x == 0) {
       ctl->head.v = 0;
@@ -213,6 +214,19 @@ int finish_queue(Part& p, cudaStream_t s, atos_stats* st, const char* what) {
   ATOS_CUDA(cudaStreamSynchronize(s));
   ATOS_CUDA(cudaGetLastError());
   const uint32_t status = (uint32_t)h->status.v;
+  if ((status || h->done.v != h->tail.v) && getenv("ATOS_DEBUG")) {
+    fprintf(stderr, "[atos debug] %s: status=%u head=%llu tail=%llu done=%llu big_count=%lld pops=%llu\n", what,
+            status, (unsigned long long)h->head.v, (unsigned long long)h->tail.v, (unsigned long long)h->done.v,
+            (long long)h->big_count.v, (unsigned long long)h->stat_pops.v);
+    if (p.big.p) {
+      std::vector<BigTask> tb(kBigSlots);
+      cudaMemcpy(tb.data(), p.big.p, sizeof(BigTask) * kBigSlots, cudaMemcpyDeviceToHost);
+      for (uint32_t i = 0; i < kBigSlots; ++i)
+        if (tb[i].state)
+          fprintf(stderr, "  slot %u state=%u gen=%u nchunks=%u next=%u finished=%u deg=%u\n", i, tb[i].state,
+                  big_gen(tb[i].ctr), big_nchunks(tb[i].ctr), big_next(tb[i].ctr), tb[i].finished, tb[i].deg);
+    }
+  }
   if (status & kStatusOverflow) {
     p.ring_clean = false;
     set_error("%s: queue overflow (ring of %llu slots lapped an unconsumed slot)", what,

@@ -9,24 +9,31 @@ namespace atos {
 //   pop v, d = depth[v]; for each neighbour w: old = atomicMin(depth+w, d+1);
 //   if d+1 < old: push w.
 // B200 additions:
-//   * prefilter: a plain load of depth[w] first; depth only decreases, so a
-//     stale value is an upper bound and `cur <= d+1` safely skips the atomic;
-//   * dedupe (optional): in-queue bitmap; the activator sets the bit with a
-//     release RMW after its atomicMin and pushes only if the bit was clear;
-//     the popper clears it with an acquire RMW BEFORE reading depth[v], so
-//     every improvement after that read re-queues v (no update is lost).
-//   * shadow depth (B200 addition): a u8 copy
-//     min(depth, 254) with 255 = "unvisited or >= 255", n bytes (67 MB at
-//     scale 26) -- small enough to stay in the 126 MB L2 (loads evict_last,
-//     the col stream evict_first), so the per-edge prefilter almost never
-//     touches HBM.  Written after a successful atomicMin; concurrent writers
-//     can only leave a value depth[w] once held, so it stays an upper bound.
+//   * shadow depth: a u8 copy min(depth, 254) with 255 = "unvisited or >= 255",
+//     n bytes (67 MB at scale 26) -- small enough to stay in the 126 MB L2
+//     (loads evict_last, the col stream evict_first), so the per-edge
+//     prefilter almost never touches HBM.  Written after a successful update;
+//     concurrent writers can only leave a value depth[w] once held, so it
+//     stays an upper bound and `shadow <= d+1` safely skips the edge;
+//   * dedupe (default): the "queued" flag lives in bit 31 of the depth word
+//     (word = depth | INQ; 0xFFFFFFFF = unreached).  The activator improves
+//     depth and sets INQ in ONE CAS and pushes only if INQ was clear; the
+//     popper clears INQ with an acquire RMW that also returns the current
+//     depth -- one location, so every improvement after the pop re-queues v
+//     and no update is lost, without release fences or a separate bitmap.
+//     At termination every queued vertex was popped, so all INQ bits are 0.
+//   * two-phase relax (pre: prefilter load, post: decision + atomics) so the
+//     engine can keep several edges' loads in flight per thread.
+constexpr uint32_t kInq = 0x80000000u;
+constexpr uint32_t kDepthMask = 0x7FFFFFFFu;
+
 struct BfsApp {
   using Payload = uint32_t;  // d + 1
+  using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
   const uint32_t* __restrict__ row_ptr;
   const uint32_t* __restrict__ col;
   uint32_t* depth;
-  uint32_t* inq;      // nullptr -> paper-literal push on every improvement
+  int dedupe;         // 0 -> paper-literal push on every improvement (atomicMin)
   uint8_t* shadow;    // nullptr -> prefilter on depth[] itself
   unsigned long long pol_first, pol_last;
 
@@ -37,35 +44,57 @@ struct BfsApp {
   }
 
   __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
-    if (inq) atom_and_acquire(inq + (v >> 5), ~(1u << (v & 31)));
-    const uint32_t d = ld_relaxed(depth + v);  // coherent read (L2): the value that caused the push
     start = __ldg(row_ptr + v);
-    deg = __ldg(row_ptr + v + 1) - start;
+    const uint32_t end = __ldg(row_ptr + v + 1);
+    uint32_t d;
+    if (dedupe) d = atom_and_acquire(depth + v, ~kInq) & kDepthMask;
+    else d = ld_relaxed(depth + v);  // coherent read (L2): the value that caused the push
+    deg = end - start;
     p = d + 1;
     return deg != 0;
   }
 
-  __device__ __forceinline__ bool relax(const Payload nd, uint32_t w, uint32_t& out) const {
-    bool need_depth_check = true;
+  __device__ __forceinline__ Token pre(const Payload nd, uint32_t w) const {
+    if (shadow) return ld_u8_hint(shadow + w, pol_last);
+    uint32_t cur;
+    asm volatile("ld.global.u32 %0, [%1];" : "=r"(cur) : "l"(depth + w));
+    return cur;
+  }
+
+  __device__ __forceinline__ bool post(const Payload nd, uint32_t w, Token tok, uint32_t& out) const {
+    uint32_t expect = 0xFFFFFFFFu;  // guess: unvisited
     if (shadow) {
-      const uint32_t sh = ld_u8_hint(shadow + w, pol_last);
-      if (sh != 255u && sh <= nd) return false;
-      need_depth_check = nd >= 255u;  // sh == 255 && nd < 255: unvisited or deeper -> must improve
+      if (tok != 255u && tok <= nd) return false;
+      if (nd >= 255u) {  // shadow carries no information at this depth: prefilter on the word
+        asm volatile("ld.global.u32 %0, [%1];" : "=r"(expect) : "l"(depth + w));
+        if (expect != 0xFFFFFFFFu && (expect & kDepthMask) <= nd) return false;
+      }
+    } else {
+      expect = tok;
+      if (expect != 0xFFFFFFFFu && (expect & kDepthMask) <= nd) return false;
     }
-    if (need_depth_check) {
-      uint32_t cur;
-      asm volatile("ld.global.u32 %0, [%1];" : "=r"(cur) : "l"(depth + w));
-      if (cur <= nd) return false;
+    bool pushed;
+    if (dedupe) {
+      while (true) {
+        const uint32_t old = atomicCAS(depth + w, expect, nd | kInq);
+        if (old == expect) {
+          pushed = (old == 0xFFFFFFFFu) || !(old & kInq);
+          break;
+        }
+        if (old != 0xFFFFFFFFu && (old & kDepthMask) <= nd) return false;
+        expect = old;
+      }
+    } else {
+      if (atomicMin(depth + w, nd) <= nd) return false;
+      pushed = true;
     }
-    const uint32_t old = atomicMin(depth + w, nd);
-    if (old <= nd) return false;
     if (shadow) st_u8_hint(shadow + w, nd < 255u ? nd : 255u, pol_last);
-    if (inq) {
-      const uint32_t bit = 1u << (w & 31);
-      if (atom_or_release(inq + (w >> 5), bit) & bit) return false;
-    }
     out = w;
-    return true;
+    return pushed;
+  }
+
+  __device__ __forceinline__ bool relax(const Payload nd, uint32_t w, uint32_t& out) const {
+    return post(nd, w, pre(nd, w), out);
   }
 };
 
@@ -87,6 +116,7 @@ struct PrApp {
   double* res;
   double alpha, eps;
   int activate;  // 1: crossing activation (default); 0: sweep-only (Check_Size variant)
+  uint32_t* dbg_expand;  // debug: per-vertex count of expanding pops
 
   __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
     const double rho = __longlong_as_double(
@@ -95,17 +125,22 @@ struct PrApp {
     start = __ldg(row_ptr + v);
     deg = __ldg(row_ptr + v + 1) - start;
     if (deg == 0 || rho == 0.0) return false;  // dangling: absorb (R-PR-3)
+    if (dbg_expand) atomicAdd(dbg_expand + v, 1u);
     p = alpha * rho / (double)deg;
     return true;
   }
 
-  __device__ __forceinline__ bool relax(const Payload delta, uint32_t w, uint32_t& out) const {
-    const double old = atomicAdd(res + w, delta);
+  using Token = double;  // residue before our atomicAdd
+  __device__ __forceinline__ Token pre(const Payload delta, uint32_t w) const { return atomicAdd(res + w, delta); }
+  __device__ __forceinline__ bool post(const Payload delta, uint32_t w, Token old, uint32_t& out) const {
     if (activate && old <= eps && old + delta > eps) {
       out = w;
       return true;
     }
     return false;
+  }
+  __device__ __forceinline__ bool relax(const Payload delta, uint32_t w, uint32_t& out) const {
+    return post(delta, w, pre(delta, w), out);
   }
 };
 

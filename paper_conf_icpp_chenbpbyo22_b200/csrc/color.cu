@@ -534,6 +534,9 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   P.fetch = (uint32_t)r.fetch;
   P.watchdog_ns = r.watchdog_ns;
   P.h0 = P.t0 = 0;
+  P.timeout_ns = r.timeout_s > 0 ? (unsigned long long)(r.timeout_s * 1e9) : 0ull;
+  P.dbg_edge = nullptr;
+  P.dbg_claim = nullptr;
   P.tl = r.timeline;
   P.tl_cap = r.timeline_cap;
   P.tl_interval_ns = r.timeline_interval_ns;

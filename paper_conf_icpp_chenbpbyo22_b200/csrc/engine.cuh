@@ -33,6 +33,7 @@
 namespace atos {
 
 enum { MODE_CTA = 0, MODE_WARP = 1, MODE_THREAD = 2 };
+constexpr int kU = 4;  // edges in flight per thread per expand iteration
 
 // ------------------------------------------------------------ big-task assist
 // A popped vertex whose degree exceeds big_threshold is not expanded by the
@@ -45,13 +46,20 @@ enum { MODE_CTA = 0, MODE_WARP = 1, MODE_THREAD = 2 };
 // popped item counts as done only when its last chunk finishes, so the
 // queue's termination rule is unchanged.  (DESIGN.md "Big-task assist".)
 struct __align__(64) BigTask {
-  unsigned long long ctr;      // (generation << 32) | next chunk
+  unsigned long long ctr;      // gen:24 | nchunks:20 | next:20 -- one word, so a claim's validity
+                               // (next < nchunks of the same generation) comes from ONE atomic
   unsigned long long payload;  // Payload bits
-  uint32_t state;              // 0 free, 1 filling, 2 active
-  uint32_t gen;
-  uint32_t v, start, deg, nchunks, finished, pad;
-  unsigned long long pad2[2];
+  uint32_t state;              // 0 free, 1 filling, 2 active (gates registration; a hint for claimers)
+  uint32_t start, deg, chunk, finished;
+  uint32_t pad[9];
 };
+constexpr uint32_t kBigNextBits = 20, kBigChunkBits = 20;
+__host__ __device__ constexpr unsigned long long big_pack(uint32_t gen, uint32_t nchunks, uint32_t next) {
+  return ((unsigned long long)(gen & 0xFFFFFFu) << 40) | ((unsigned long long)nchunks << 20) | next;
+}
+__host__ __device__ constexpr uint32_t big_gen(unsigned long long c) { return (uint32_t)(c >> 40); }
+__host__ __device__ constexpr uint32_t big_nchunks(unsigned long long c) { return (uint32_t)(c >> 20) & 0xFFFFFu; }
+__host__ __device__ constexpr uint32_t big_next(unsigned long long c) { return (uint32_t)c & 0xFFFFFu; }
 
 struct EngineParams {
   Ring q;
@@ -62,6 +70,9 @@ struct EngineParams {
   uint32_t nbig, big_threshold, big_chunk;
   unsigned long long* tl;           // progress timeline (nullptr: off)
   uint32_t tl_cap, tl_interval_ns;
+  unsigned long long timeout_ns;    // cfg.timeout_s as a device deadline (0: none) -- catches livelock
+  uint32_t* dbg_edge;               // debug (ATOS_DEBUG_EDGES): per-edge relaxation counts
+  uint32_t* dbg_claim;              // debug: last gen that claimed (slot, chunk), 64 x 4096
 };
 
 // Progress sample (globaltimer, done, tail, head) at most every tl_interval_ns,
@@ -98,46 +109,63 @@ __device__ __forceinline__ Payload payload_from(unsigned long long b) {
   return p;
 }
 
+__device__ __forceinline__ unsigned long long atom_add_acquire(unsigned long long* p, unsigned long long v) {
+  unsigned long long old;
+  asm volatile("atom.acquire.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+  return old;
+}
+__device__ __forceinline__ unsigned long long atom_exch_release(unsigned long long* p, unsigned long long v) {
+  unsigned long long old;
+  asm volatile("atom.release.gpu.global.exch.b64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+  return old;
+}
+
 // Register item v (row [start, start+deg), payload p) as a big task.  False
-// when no free slot was found (the caller expands the vertex itself).
-// Order: state 0->1 (CAS) ; fields ; gen+1 (atomic) ; ctr = gen<<32 ; state = 2.
+// when the chosen slot is busy (the caller expands the vertex itself).
+// The fields and `finished` are written first; ONE release exchange then
+// publishes (gen+1, nchunks, next=0) in the counter word.  Chunk size is
+// raised if needed so nchunks < 2^19 (the counter's 20-bit field keeps room
+// for stale over-claims).
 template <class Payload>
 __device__ __forceinline__ bool register_big(const EngineParams& P, uint32_t v, uint32_t start, uint32_t deg,
                                              const Payload& p) {
   const uint32_t slot = (uint32_t)(atomicAdd(&P.q.ctl->big_rr.v, 1ull) % P.nbig);
   BigTask* t = P.big + slot;
   if (atomicCAS(&t->state, 0u, 1u) != 0u) return false;
-  t->v = v;
+  fence_acq_rel_gpu();  // the previous instance's retirement happens-before our writes
+  uint32_t chunk = P.big_chunk;
+  const uint32_t minchunk = (deg + (1u << 19) - 1) >> 19;
+  if (chunk < minchunk) chunk = minchunk;
+  const uint32_t nchunks = (deg + chunk - 1) / chunk;
   t->start = start;
   t->deg = deg;
-  t->nchunks = (deg + P.big_chunk - 1) / P.big_chunk;
+  t->chunk = chunk;
   t->finished = 0;
   t->payload = payload_bits(p);
-  const uint32_t gen = atomicAdd(&t->gen, 1u) + 1u;  // RMW: monotone, never a stale read
-  __threadfence();
-  atomicExch(&t->ctr, (unsigned long long)gen << 32);
-  __threadfence();
-  atomicExch(&t->state, 2u);
+  const uint32_t gen = big_gen(ld_relaxed(&t->ctr)) + 1u;  // we own the slot: only `next` moves meanwhile
+  atom_exch_release(&t->ctr, big_pack(gen, nchunks, 0));
+  st_release(&t->state, 2u);
   atomicAdd(&P.q.ctl->big_count.v, 1ull);
   return true;
 }
 
 // Warp-collective: claim one chunk of an active big task.  Returns the slot
 // (or -1) and sets chunk; every lane gets the same answer.  When a chunk is
-// claimed, lane 0 (which performed the acquire) writes the task fields to
-// out[0..3] = start, deg, payload lo, payload hi (shared memory).
-// A counter increment is valid only if, once the slot is active again, the
-// slot's generation still equals the one carried by the counter value and the
-// chunk index is in range -- so late claims on a retired/reused slot are
-// rejected and no chunk is ever processed twice.
+// claimed, lane 0 writes out[0..5] = start, deg, payload lo, payload hi,
+// nchunks, chunk size (shared memory).  A claim is valid iff the counter value
+// returned by the acquire RMW has next < nchunks: a valid chunk keeps its
+// task instance alive (it cannot retire before the chunk finishes), so the
+// fields read after the acquire are that instance's; stale over-claims on a
+// retired or refilling slot see next >= nchunks and are dropped.
 __device__ __forceinline__ int claim_big_warp(const EngineParams& P, uint32_t& chunk, uint32_t* out) {
   if (ld_relaxed(&P.q.ctl->big_count.v) == 0) return -1;
   for (uint32_t base = 0; base < P.nbig; base += 32) {
     const uint32_t i = base + lane_id();
     bool act = false;
     if (i < P.nbig) {
-      const BigTask* t = P.big + i;
-      act = ld_relaxed(&t->state) == 2u && (uint32_t)ld_relaxed(&t->ctr) < ld_relaxed(&t->nchunks);
+      BigTask* t = P.big + i;
+      const unsigned long long c = ld_relaxed(&t->ctr);
+      act = ld_relaxed(&t->state) == 2u && big_next(c) < big_nchunks(c);
     }
     unsigned m = __ballot_sync(0xffffffffu, act);
     while (m) {
@@ -147,21 +175,22 @@ __device__ __forceinline__ int claim_big_warp(const EngineParams& P, uint32_t& c
       int ok = 0;
       uint32_t c = 0;
       if (lane_id() == 0) {
-        const unsigned long long old = atomicAdd(&t->ctr, 1ull);
-        const uint32_t gen = (uint32_t)(old >> 32);
-        c = (uint32_t)old;
-        uint32_t st = ld_acquire(&t->state);
-        while (st == 1u) {  // a registration is filling the slot: wait for it to settle
-          __nanosleep(32);
-          st = ld_acquire(&t->state);
-        }
-        if (st == 2u && ld_relaxed(&t->gen) == gen && c < ld_relaxed(&t->nchunks)) {
+        const unsigned long long old = atom_add_acquire(&t->ctr, 1ull);
+        c = big_next(old);
+        if (c < big_nchunks(old)) {
           ok = 1;
           out[0] = ld_relaxed(&t->start);
           out[1] = ld_relaxed(&t->deg);
           const unsigned long long pb = ld_relaxed(&t->payload);
           out[2] = (uint32_t)pb;
           out[3] = (uint32_t)(pb >> 32);
+          out[4] = big_nchunks(old);
+          out[5] = ld_relaxed(&t->chunk);
+          if (P.dbg_claim && c < 4096) {
+            const uint32_t prev = atomicExch(P.dbg_claim + (base + L) * 4096 + c, big_gen(old));
+            if (prev == big_gen(old))
+              printf("DUP claim slot %u gen %u chunk %u\n", base + L, big_gen(old), c);
+          }
         }
       }
       ok = __shfl_sync(0xffffffffu, ok, 0);
@@ -176,14 +205,17 @@ __device__ __forceinline__ int claim_big_warp(const EngineParams& P, uint32_t& c
 }
 
 // A chunk is finished (its pushes published): the last finisher retires the
-// task and counts the original item as done.
-__device__ __forceinline__ void finish_big_chunk(const EngineParams& P, int slot) {
+// task and counts the original item as done.  `nchunks` is the value from the
+// claim: once our increment lands the slot may be retired and refilled, so
+// nothing of the slot is re-read after it.
+__device__ __forceinline__ void finish_big_chunk(const EngineParams& P, int slot, uint32_t nchunks) {
   BigTask* t = P.big + slot;
   fence_acq_rel_gpu();
   const uint32_t f = atomicAdd(&t->finished, 1u);
-  if (f + 1 == ld_relaxed(&t->nchunks)) {
+  if (P.dbg_claim && f >= nchunks) printf("OVERFINISH slot %d f %u nchunks %u\n", slot, f, nchunks);
+  if (f + 1 == nchunks) {
     fence_acq_rel_gpu();
-    atomicExch(&t->state, 0u);
+    st_release(&t->state, 0u);
     atomicAdd(&P.q.ctl->big_count.v, (unsigned long long)-1ll);
     atom_add_release(&P.q.ctl->done.v, 1ull);
   }
@@ -204,9 +236,9 @@ struct GroupSmem {
 
 template <class Payload>
 __host__ __device__ constexpr size_t group_smem_bytes(uint32_t K) {
-  // 3 u32 arrays, payload array, two u64 pending arrays, 48 u32 counters
+  // 3 u32 arrays, payload array, two u64 pending arrays, 56 u32 counters
   return ((size_t)K * (3 * sizeof(uint32_t)) + 15) / 16 * 16 + ((size_t)K * sizeof(Payload) + 15) / 16 * 16 +
-         (size_t)K * 16 + 48 * sizeof(uint32_t);
+         (size_t)K * 16 + 56 * sizeof(uint32_t);
 }
 
 template <class Payload>
@@ -266,6 +298,7 @@ struct Worker {
   bool first;
   unsigned backoff;
   unsigned long long idle_since;
+  unsigned long long deadline;
 
   __device__ __forceinline__ void init(unsigned char* arena, const EngineParams& P) {
     const uint32_t nwarps = blockDim.x >> 5;
@@ -279,6 +312,7 @@ struct Worker {
     first = true;
     backoff = 32;
     idle_since = 0;
+    deadline = P.timeout_ns ? globaltimer() + P.timeout_ns : 0;
     if (r == 0) s.ctr[1] = 0;
     group_sync<MODE>();
   }
@@ -292,7 +326,11 @@ struct Worker {
       if (r == 0) {
         s.ctr[0] = 0; s.ctr[2] = 0; s.ctr[3] = 0; s.ctr[4] = 0; s.ctr[5] = 0;
         *(unsigned long long*)&s.ctr[6] = 0;
-        if (!PERSIST) {
+        if (deadline && globaltimer() > deadline) {
+          // busy past cfg.timeout_s (e.g. a livelocking policy): stop everyone
+          atomicOr((unsigned int*)&q.ctl->status.v, kStatusTimeout);
+          s.ctr[3] = 1;
+        } else if (!PERSIST) {
           if (!first) {
             s.ctr[3] = 1;
           } else {
@@ -428,21 +466,34 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
       const int slot = (int)s.ctr[41];
       if (slot >= 0) {
         const uint32_t c = s.ctr[42];
-        const uint32_t b0 = c * P.big_chunk;
-        const uint32_t len = min(P.big_chunk, s.ctr[44] - b0);
+        const uint32_t b0 = c * s.ctr[48];
+        const uint32_t len = min(s.ctr[48], s.ctr[44] - b0);
         const uint32_t st0 = s.ctr[43] + b0;
         const Payload p = payload_from<Payload>(((unsigned long long)s.ctr[46] << 32) | s.ctr[45]);
         my_edges += (r == 0) ? len : 0;
-        for (uint32_t base = 0; base < len; base += G) {
-          const uint32_t e = base + r;
-          bool want = false;
-          uint32_t out = 0;
-          if (e < len) want = app.relax(p, app.neighbor(st0 + e), out);
-          pusher.push(q, want, out, P.watchdog_ns);
+        for (uint32_t base = 0; base < len; base += G * kU) {
+          uint32_t w[kU];
+          typename App::Token tk[kU];
+#pragma unroll
+          for (int k = 0; k < kU; ++k)
+            if (base + k * G + r < len) {
+              w[k] = app.neighbor(st0 + base + k * G + r);
+              if (P.dbg_edge) atomicAdd(P.dbg_edge + st0 + base + k * G + r, 1u);
+            }
+#pragma unroll
+          for (int k = 0; k < kU; ++k)
+            if (base + k * G + r < len) tk[k] = app.pre(p, w[k]);
+#pragma unroll
+          for (int k = 0; k < kU; ++k) {
+            bool want = false;
+            uint32_t out = 0;
+            if (base + k * G + r < len) want = app.post(p, w[k], tk[k], out);
+            pusher.push(q, want, out, P.watchdog_ns);
+          }
         }
         pusher.flush(q, P.watchdog_ns);
         group_sync<MODE>();
-        if (r == 0) finish_big_chunk(P, slot);
+        if (r == 0) finish_big_chunk(P, slot, s.ctr[47]);
         group_sync<MODE>();
         continue;
       }
@@ -480,35 +531,70 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
       for (uint32_t i = i0; i < i1; ++i) { const uint32_t d = s.off[i]; s.off[i] = excl; excl += d; }
       __syncthreads();
       my_edges += (r == 0) ? total : 0;
-      for (uint32_t base = 0; base < total; base += G) {
-        const uint32_t e = base + r;
-        bool want = false;
-        uint32_t out = 0;
-        if (e < total) {
-          // largest i with off[i] <= e
-          uint32_t lo = 0, hi = nready;
-          while (hi - lo > 1) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (s.off[mid] <= e) lo = mid; else hi = mid;
+      // kU edges per thread per iteration (strided by G: each k is a coalesced
+      // warp access); all col loads, then all prefilter loads, then the
+      // decisions/atomics -- kU independent memory chains in flight per thread.
+      for (uint32_t base = 0; base < total; base += G * kU) {
+        uint32_t lo[kU], w[kU];
+        typename App::Token tk[kU];
+        uint32_t from = 0;
+#pragma unroll
+        for (int k = 0; k < kU; ++k) {
+          const uint32_t e = base + k * G + r;
+          lo[k] = 0xFFFFFFFFu;
+          if (e < total) {
+            // largest i >= from with off[i] <= e (owners are monotone in k)
+            uint32_t l = from, h = nready;
+            while (h - l > 1) {
+              const uint32_t mid = (l + h) >> 1;
+              if (s.off[mid] <= e) l = mid; else h = mid;
+            }
+            lo[k] = l;
+            from = l;
           }
-          const uint32_t w = app.neighbor(s.start[lo] + (e - s.off[lo]));
-          want = app.relax(s.pay[lo], w, out);
         }
-        pusher.push(q, want, out, P.watchdog_ns);
+#pragma unroll
+        for (int k = 0; k < kU; ++k)
+          if (lo[k] != 0xFFFFFFFFu) {
+            const uint32_t e = s.start[lo[k]] + (base + k * G + r - s.off[lo[k]]);
+            w[k] = app.neighbor(e);
+            if (P.dbg_edge) atomicAdd(P.dbg_edge + e, 1u);
+          }
+#pragma unroll
+        for (int k = 0; k < kU; ++k)
+          if (lo[k] != 0xFFFFFFFFu) tk[k] = app.pre(s.pay[lo[k]], w[k]);
+#pragma unroll
+        for (int k = 0; k < kU; ++k) {
+          bool want = false;
+          uint32_t out = 0;
+          if (lo[k] != 0xFFFFFFFFu) want = app.post(s.pay[lo[k]], w[k], tk[k], out);
+          pusher.push(q, want, out, P.watchdog_ns);
+        }
       }
     } else if (MODE == MODE_WARP) {
       for (uint32_t k = 0; k < nready; ++k) {
         const uint32_t st = s.start[k], dg = s.off[k];
         const Payload p = s.pay[k];
         my_edges += (r == 0) ? dg : 0;
-        for (uint32_t j = 0; j < dg; j += 32) {
-          bool want = false;
-          uint32_t out = 0;
-          if (j + r < dg) {
-            const uint32_t w = app.neighbor(st + j + r);
-            want = app.relax(p, w, out);
+        for (uint32_t j = 0; j < dg; j += 32 * kU) {
+          uint32_t w[kU];
+          typename App::Token tk[kU];
+#pragma unroll
+          for (int k = 0; k < kU; ++k)
+            if (j + k * 32 + r < dg) {
+              w[k] = app.neighbor(st + j + k * 32 + r);
+              if (P.dbg_edge) atomicAdd(P.dbg_edge + st + j + k * 32 + r, 1u);
+            }
+#pragma unroll
+          for (int k = 0; k < kU; ++k)
+            if (j + k * 32 + r < dg) tk[k] = app.pre(p, w[k]);
+#pragma unroll
+          for (int k = 0; k < kU; ++k) {
+            bool want = false;
+            uint32_t out = 0;
+            if (j + k * 32 + r < dg) want = app.post(p, w[k], tk[k], out);
+            pusher.push(q, want, out, P.watchdog_ns);
           }
-          pusher.push(q, want, out, P.watchdog_ns);
         }
       }
     } else {

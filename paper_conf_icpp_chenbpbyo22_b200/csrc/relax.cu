@@ -1,11 +1,16 @@
 // relax.cu -- single-partition BFS and PageRank: init kernels, launchers
 // (persistent and discrete), finalisation.
 #include <algorithm>
+#include <cstdlib>
+#include <vector>
 
-#include "apps.cuh"
 #include "internal.h"
+#include "apps.cuh"
 
 namespace atos {
+
+static uint32_t* g_dbg_edge = nullptr;  // debug (ATOS_DEBUG_EDGES): per-edge relaxation counts
+static uint32_t* g_dbg_claim = nullptr;
 
 // ------------------------------------------------------------- init kernels
 // Start of a run on a persistent ring: abandon stale over-claims (head = tail),
@@ -38,13 +43,12 @@ __global__ void k_run_begin(QueueCtl* ctl) {
 
 // BFS init (Alg.1 P:721-725 "vertex.dist = MAX_UINT32", frontier = [source];
 // source depth 0, R-BFS-1).  depth[] was memset to 0xFF on the stream.
-__global__ void k_bfs_init(uint32_t* depth, uint32_t* inq, uint8_t* shadow, Ring q, uint32_t src,
+__global__ void k_bfs_init(uint32_t* depth, int dedupe, uint8_t* shadow, Ring q, uint32_t src,
                            unsigned long long wd) {
   if (threadIdx.x == 0 && blockIdx.x == 0) {
     run_begin(q.ctl);
-    depth[src] = 0;
+    depth[src] = dedupe ? kInq : 0u;  // depth 0, queued
     if (shadow) shadow[src] = 0;
-    if (inq) inq[src >> 5] |= 1u << (src & 31);
     const unsigned long long idx = q.ctl->tail.v;
     q.ctl->tail.v = idx + 1;
     publish_one(q, idx, src, wd);
@@ -240,6 +244,9 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
   const int block = mode == MODE_CTA ? r.worker : r.block_threads;
   // hub assist (persistent CTA / warp workers): auto threshold = 32 edges per
   // worker thread, chunks of 8 edges per worker thread (>= 1024)
+  P.timeout_ns = r.timeout_s > 0 ? (unsigned long long)(r.timeout_s * 1e9) : 0ull;
+  P.dbg_edge = g_dbg_edge;
+  P.dbg_claim = g_dbg_claim;
   P.tl = r.timeline;
   P.tl_cap = r.timeline_cap;
   P.tl_interval_ns = r.timeline_interval_ns;
@@ -274,22 +281,16 @@ int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolve
   uint64_t want = r.queue_capacity ? r.queue_capacity : (uint64_t)std::max<int64_t>(2 * n, 1024);
   if (!r.dedupe && !r.queue_capacity) want = (uint64_t)std::max<int64_t>(4 * n, 4096);
   ATOS_TRY(ensure_queue(p, pow2_at_least(want), s));
-  uint32_t* inq = nullptr;
-  if (r.dedupe) {
-    ATOS_TRY(p.bitmap.ensure(((size_t)n + 31) / 32 * 4));
-    inq = p.bitmap.as<uint32_t>();
-    ATOS_CUDA(cudaMemsetAsync(inq, 0, ((size_t)n + 31) / 32 * 4, s));
-  }
   ATOS_CUDA(cudaMemsetAsync(depth, 0xFF, (size_t)n * 4, s));
   ATOS_TRY(p.shadow.ensure((size_t)n));
   uint8_t* shadow = p.shadow.as<uint8_t>();
   ATOS_CUDA(cudaMemsetAsync(shadow, 0xFF, (size_t)n, s));
   Ring q = ring_of(p);
-  k_bfs_init<<<1, 32, 0, s>>>(depth, inq, shadow, q, (uint32_t)src, r.watchdog_ns);
+  k_bfs_init<<<1, 32, 0, s>>>(depth, r.dedupe, shadow, q, (uint32_t)src, r.watchdog_ns);
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, depth, (size_t)n * 4, true);
-  BfsApp app{p.row_ptr, p.col, depth, inq, shadow, 0ull, 0ull};
+  BfsApp app{p.row_ptr, p.col, depth, r.dedupe, shadow, 0ull, 0ull};
   p.ring_clean = false;
   int rc = launch_relax(app, q, r, p, st);
   if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
@@ -323,7 +324,20 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, res, (size_t)n * 8, true);
-  PrApp app{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, r.check_size > 0 ? 0 : 1};
+  PrApp app{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, r.check_size > 0 ? 0 : 1, nullptr};
+  uint32_t* dbg_edge = nullptr;
+  const bool dbg = getenv("ATOS_DEBUG_EDGES") != nullptr;
+  if (dbg) {
+    ATOS_CUDA(cudaMalloc(&dbg_edge, (size_t)p.m_local * 4 + 4));
+    ATOS_CUDA(cudaMalloc(&app.dbg_expand, (size_t)n * 4 + 4));
+    ATOS_CUDA(cudaMemset(dbg_edge, 0, (size_t)p.m_local * 4 + 4));
+    ATOS_CUDA(cudaMemset(app.dbg_expand, 0, (size_t)n * 4 + 4));
+    g_dbg_edge = dbg_edge;
+    if (!g_dbg_claim) {
+      cudaMalloc(&g_dbg_claim, 64 * 4096 * 4);
+      cudaMemset(g_dbg_claim, 0, 64 * 4096 * 4);
+    }
+  }
   p.ring_clean = false;
   int rc = ATOS_OK;
   if (r.check_size <= 0) {
@@ -350,6 +364,32 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
     }
   }
   if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
+  g_dbg_edge = nullptr;
+  if (dbg) {
+    g_dbg_claim = g_dbg_claim;  // kept across calls (generations keep increasing)
+    cudaDeviceSynchronize();
+    std::vector<uint32_t> ec(p.m_local), xc(n), rp(n + 1);
+    cudaMemcpy(ec.data(), dbg_edge, p.m_local * 4, cudaMemcpyDeviceToHost);
+    cudaMemcpy(xc.data(), app.dbg_expand, n * 4, cudaMemcpyDeviceToHost);
+    cudaMemcpy(rp.data(), p.row_ptr, (n + 1) * 4, cudaMemcpyDeviceToHost);
+    long over = 0, under = 0, vbad = 0;
+    for (int64_t v = 0; v < n; ++v) {
+      bool b = false;
+      for (uint32_t e = rp[v]; e < rp[v + 1]; ++e) {
+        if (ec[e] > xc[v]) { ++over; b = true; }
+        if (ec[e] < xc[v]) { ++under; b = true; }
+      }
+      if (b && vbad < 8) {
+        fprintf(stderr, "  v=%lld deg=%u expands=%u edge counts:", (long long)v, rp[v + 1] - rp[v], xc[v]);
+        for (uint32_t e = rp[v]; e < rp[v + 1] && e < rp[v] + 24; ++e) fprintf(stderr, " %u", ec[e]);
+        fprintf(stderr, "\n");
+      }
+      vbad += b;
+    }
+    fprintf(stderr, "[atos debug edges] over=%ld under=%ld bad_vertices=%ld\n", over, under, vbad);
+    cudaFree(dbg_edge);
+    cudaFree(app.dbg_expand);
+  }
   if (rc != ATOS_OK) return rc;
   ATOS_CUDA(cudaMemsetAsync(sum, 0, 8, s));
   k_pr_finalize<<<gs, 256, 0, s>>>(rank, res, n, sum);
