@@ -119,10 +119,10 @@ __global__ void __launch_bounds__(1024) k_color_warp(ColorCtx c, EngineParams P)
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const uint32_t nwarps = blockDim.x >> 5;
   uint32_t* pushbuf = (uint32_t*)smem_raw;
-  uint32_t* bms = pushbuf + nwarps * 64;  // 32 words per warp
+  uint32_t* bms = pushbuf + nwarps * kPushBuf;  // 32 words per warp
   Worker<MODE_WARP, PERSIST, uint32_t> wk;
   wk.init((unsigned char*)(bms + nwarps * 32), P);
-  WarpPusher pusher{pushbuf + warp_id() * 64, 0, 0};
+  WarpPusher pusher = make_pusher(pushbuf);
   unsigned long long pops = 0, edges = 0;
   while (true) {
     const uint32_t nready = wk.acquire(P);
@@ -147,14 +147,14 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
   const uint32_t nwarps = blockDim.x >> 5;
   const uint32_t F = P.fetch;
   uint32_t* pushbuf = (uint32_t*)smem_raw;
-  uint32_t* wbm = pushbuf + nwarps * 64;   // 32 words per warp (fallback windows)
+  uint32_t* wbm = pushbuf + nwarps * kPushBuf;   // 32 words per warp (fallback windows)
   uint32_t* ibm = wbm + nwarps * 32;       // 32 words per item
   uint32_t* flag = ibm + F * 32;           // per item: check found a self-conflict
   int32_t* cval = (int32_t*)(flag + F);    // per item: colour of v (check items)
   Worker<MODE_CTA, PERSIST, uint32_t> wk;
   wk.init((unsigned char*)(cval + F), P);
   const GroupSmem<uint32_t>& s = wk.s;
-  WarpPusher pusher{pushbuf + warp_id() * 64, 0, 0};
+  WarpPusher pusher = make_pusher(pushbuf);
   unsigned long long pops = 0, edges = 0;
   const uint32_t tid = threadIdx.x, B = blockDim.x;
   while (true) {
@@ -279,9 +279,9 @@ __global__ void __launch_bounds__(1024) k_color_thread(ColorCtx c, EngineParams 
   const uint32_t nwarps = blockDim.x >> 5;
   uint32_t* pushbuf = (uint32_t*)smem_raw;
   Worker<MODE_THREAD, PERSIST, uint32_t> wk;
-  wk.init((unsigned char*)(pushbuf + nwarps * 64), P);
+  wk.init((unsigned char*)(pushbuf + nwarps * kPushBuf), P);
   const GroupSmem<uint32_t>& s = wk.s;
-  WarpPusher pusher{pushbuf + warp_id() * 64, 0, 0};
+  WarpPusher pusher = make_pusher(pushbuf);
   unsigned long long pops = 0, edges = 0;
   const uint32_t lane = lane_id();
   while (true) {
@@ -550,17 +550,17 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   wt.start(s);
   if (mode == MODE_WARP) {
     const int block = r.block_threads, nw = block / 32;
-    const size_t smem = (size_t)nw * 64 * 4 + (size_t)nw * 32 * 4 + group_smem_bytes<uint32_t>(r.fetch) * nw;
+    const size_t smem = (size_t)nw * kPushBuf * 4 + (size_t)nw * 32 * 4 + group_smem_bytes<uint32_t>(r.fetch) * nw;
     rc = launch_color_kernel(k_color_warp<true>, k_color_warp<false>, c, P, r, block, smem,
                              (uint64_t)r.fetch * nw, p, st);
   } else if (mode == MODE_CTA) {
     const int block = r.worker, nw = block / 32;
-    const size_t smem = (size_t)nw * 64 * 4 + (size_t)nw * 32 * 4 + (size_t)r.fetch * 32 * 4 +
+    const size_t smem = (size_t)nw * kPushBuf * 4 + (size_t)nw * 32 * 4 + (size_t)r.fetch * 32 * 4 +
                         (size_t)r.fetch * 8 + group_smem_bytes<uint32_t>(r.fetch);
     rc = launch_color_kernel(k_color_cta<true>, k_color_cta<false>, c, P, r, block, smem, (uint64_t)r.fetch, p, st);
   } else {
     const int block = r.block_threads, nw = block / 32;
-    const size_t smem = (size_t)nw * 64 * 4 + group_smem_bytes<uint32_t>(32u * r.fetch) * nw;
+    const size_t smem = (size_t)nw * kPushBuf * 4 + group_smem_bytes<uint32_t>(32u * r.fetch) * nw;
     rc = launch_color_kernel(k_color_thread<true>, k_color_thread<false>, c, P, r, block, smem,
                              (uint64_t)r.fetch * 32 * nw, p, st);
   }

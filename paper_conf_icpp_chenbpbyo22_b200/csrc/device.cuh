@@ -251,52 +251,72 @@ __device__ __forceinline__ int try_consume(const Ring& q, unsigned long long idx
   return 1;
 }
 
-// Per-warp staging buffer in shared memory.  push() is warp-collective (all 32
-// lanes call it with their own `want` flag); entries accumulate and are
-// published 32 at a time: one atomicAdd on tail per 32 pushes, one coalesced
-// 128-byte release store.  flush() publishes the remainder.
+// Per-warp staging ring in shared memory (kPushBuf entries).  push_n() is
+// warp-collective (all 32 lanes call it, each with up to N candidate items);
+// entries accumulate and are published 32 at a time: one atomicAdd on tail
+// per 32 pushes and one coalesced release store per lane.  flush() publishes
+// the remainder.  (The paper's push_warp, aggregated to whole lines.)
+constexpr uint32_t kPushBuf = 256;
+
 struct WarpPusher {
-  uint32_t* buf;      // 64 entries of shared memory owned by this warp
+  uint32_t* buf;      // kPushBuf entries of shared memory owned by this warp
+  uint32_t head;      // warp-uniform ring head
   uint32_t cnt;       // warp-uniform fill level (< 32 between calls)
   uint32_t total;     // warp-uniform number of pushes issued (stats)
 
   __device__ __forceinline__ void publish(const Ring& q, uint32_t k, unsigned long long watchdog_ns) {
-    // k <= 32 entries in buf[0..k)
+    // k <= 32 entries at buf[head .. head+k)
     unsigned long long base = 0;
     if (lane_id() == 0) base = atomicAdd(&q.ctl->tail.v, (unsigned long long)k);
     base = __shfl_sync(0xffffffffu, base, 0);
-    if (lane_id() < k) publish_one(q, base + lane_id(), buf[lane_id()], watchdog_ns);
+    if (lane_id() < k) publish_one(q, base + lane_id(), buf[(head + lane_id()) & (kPushBuf - 1)], watchdog_ns);
+    head = (head + k) & (kPushBuf - 1);
+    cnt -= k;
     total += k;
   }
 
-  __device__ __forceinline__ void push(const Ring& q, bool want, uint32_t item,
-                                       unsigned long long watchdog_ns) {
-    unsigned m = __ballot_sync(0xffffffffu, want);
-    if (m == 0) return;
-    uint32_t pos = cnt + __popc(m & ((1u << lane_id()) - 1u));
-    if (want) buf[pos] = item;
-    cnt += __popc(m);
+  template <int N>
+  __device__ __forceinline__ void push_n(const Ring& q, const bool (&want)[N], const uint32_t (&item)[N],
+                                         unsigned long long watchdog_ns) {
+    uint32_t c = 0;
+#pragma unroll
+    for (int k = 0; k < N; ++k) c += want[k] ? 1u : 0u;
+    uint32_t incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane_id() >= (uint32_t)o) incl += y;
+    }
+    const uint32_t sum = __shfl_sync(0xffffffffu, incl, 31);
+    if (sum == 0) return;
+    uint32_t pos = head + cnt + incl - c;
+#pragma unroll
+    for (int k = 0; k < N; ++k)
+      if (want[k]) buf[(pos++) & (kPushBuf - 1)] = item[k];
+    cnt += sum;
     __syncwarp();
-    if (cnt >= 32) {
+    while (cnt >= 32) {
       publish(q, 32, watchdog_ns);
-      __syncwarp();
-      uint32_t rest = cnt - 32;
-      uint32_t tmp = lane_id() < rest ? buf[32 + lane_id()] : 0;
-      __syncwarp();
-      if (lane_id() < rest) buf[lane_id()] = tmp;
-      cnt = rest;
       __syncwarp();
     }
   }
 
+  __device__ __forceinline__ void push(const Ring& q, bool want, uint32_t item, unsigned long long watchdog_ns) {
+    const bool w[1] = {want};
+    const uint32_t it[1] = {item};
+    push_n<1>(q, w, it, watchdog_ns);
+  }
+
   __device__ __forceinline__ void flush(const Ring& q, unsigned long long watchdog_ns) {
-    if (cnt) {
-      publish(q, cnt, watchdog_ns);
-      cnt = 0;
-    }
+    if (cnt) publish(q, cnt, watchdog_ns);
     __syncwarp();
   }
 };
+
+// the calling warp's pusher over a per-block array of kPushBuf-entry rings
+__device__ __forceinline__ WarpPusher make_pusher(uint32_t* bufs) {
+  return WarpPusher{bufs + warp_id() * kPushBuf, 0u, 0u, 0u};
+}
 
 // -------------------------------------------------------- block-wide helpers
 // exclusive scan of one value per thread; returns the exclusive prefix and

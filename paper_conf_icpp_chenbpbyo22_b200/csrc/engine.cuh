@@ -434,13 +434,13 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
   using Payload = typename App::Payload;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const uint32_t nwarps = blockDim.x >> 5;
-  // push buffers first (64 u32 per warp), then one arena per group
+  // push rings first (kPushBuf u32 per warp), then one arena per group
   uint32_t* pushbuf = (uint32_t*)smem_raw;
   Worker<MODE, PERSIST, Payload> wk;
-  wk.init(smem_raw + (size_t)nwarps * 64 * 4, P);
+  wk.init(smem_raw + (size_t)nwarps * kPushBuf * 4, P);
   const GroupSmem<Payload>& s = wk.s;
   const uint32_t r = wk.r, G = wk.G;
-  WarpPusher pusher{pushbuf + warp_id() * 64, 0, 0};
+  WarpPusher pusher = make_pusher(pushbuf);
   unsigned long long my_pops = 0, my_edges = 0;
   const Ring& q = P.q;
   app.prepare();
@@ -472,24 +472,27 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
         const Payload p = payload_from<Payload>(((unsigned long long)s.ctr[46] << 32) | s.ctr[45]);
         my_edges += (r == 0) ? len : 0;
         for (uint32_t base = 0; base < len; base += G * kU) {
+          const uint32_t j0 = base + r * kU;  // kU consecutive edges per lane
           uint32_t w[kU];
           typename App::Token tk[kU];
 #pragma unroll
           for (int k = 0; k < kU; ++k)
-            if (base + k * G + r < len) {
-              w[k] = app.neighbor(st0 + base + k * G + r);
-              if (P.dbg_edge) atomicAdd(P.dbg_edge + st0 + base + k * G + r, 1u);
+            if (j0 + k < len) {
+              w[k] = app.neighbor(st0 + j0 + k);
+              if (P.dbg_edge) atomicAdd(P.dbg_edge + st0 + j0 + k, 1u);
             }
 #pragma unroll
           for (int k = 0; k < kU; ++k)
-            if (base + k * G + r < len) tk[k] = app.pre(p, w[k]);
+            if (j0 + k < len) tk[k] = app.pre(p, w[k]);
+          bool want[kU];
+          uint32_t out[kU];
 #pragma unroll
           for (int k = 0; k < kU; ++k) {
-            bool want = false;
-            uint32_t out = 0;
-            if (base + k * G + r < len) want = app.post(p, w[k], tk[k], out);
-            pusher.push(q, want, out, P.watchdog_ns);
+            want[k] = false;
+            out[k] = 0;
+            if (j0 + k < len) want[k] = app.post(p, w[k], tk[k], out[k]);
           }
+          pusher.push_n<kU>(q, want, out, P.watchdog_ns);
         }
         pusher.flush(q, P.watchdog_ns);
         group_sync<MODE>();
@@ -531,45 +534,65 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
       for (uint32_t i = i0; i < i1; ++i) { const uint32_t d = s.off[i]; s.off[i] = excl; excl += d; }
       __syncthreads();
       my_edges += (r == 0) ? total : 0;
-      // kU edges per thread per iteration (strided by G: each k is a coalesced
-      // warp access); all col loads, then all prefilter loads, then the
-      // decisions/atomics -- kU independent memory chains in flight per thread.
+      // kU CONSECUTIVE edges per lane per iteration (a warp covers 32*kU
+      // consecutive flattened edges, so col reads stay coalesced).  Owners:
+      // lanes 0/1 binary-search the owners of the warp's first/last edge over
+      // the whole batch, then every lane searches only that narrow range and
+      // walks forward over its kU edges.  All col loads, then all prefilter
+      // loads, then the decisions/atomics: kU memory chains in flight per lane.
+      const uint32_t wspan = 32u * kU;
       for (uint32_t base = 0; base < total; base += G * kU) {
-        uint32_t lo[kU], w[kU];
+        const uint32_t wfirst = base + (r & ~31u) * kU;
+        if (wfirst >= total) continue;  // warp-uniform; no collective below is skipped by part of a warp
+        const uint32_t wlast = min(wfirst + wspan, total) - 1;
+        uint32_t ob = 0;
+        if (lane_id() < 2) {
+          const uint32_t e = lane_id() == 0 ? wfirst : wlast;
+          uint32_t l = 0, h = nready;
+          while (h - l > 1) {
+            const uint32_t mid = (l + h) >> 1;
+            if (s.off[mid] <= e) l = mid; else h = mid;
+          }
+          ob = l;
+        }
+        const uint32_t olo = __shfl_sync(0xffffffffu, ob, 0), ohi = __shfl_sync(0xffffffffu, ob, 1);
+        const uint32_t e0 = wfirst + lane_id() * kU;
+        uint32_t o = olo;
+        {
+          uint32_t l = olo, h = ohi + 1;
+          while (h - l > 1) {
+            const uint32_t mid = (l + h) >> 1;
+            if (s.off[mid] <= e0) l = mid; else h = mid;
+          }
+          o = l;
+        }
+        uint32_t w[kU], own[kU];
+        bool val[kU];
         typename App::Token tk[kU];
-        uint32_t from = 0;
 #pragma unroll
         for (int k = 0; k < kU; ++k) {
-          const uint32_t e = base + k * G + r;
-          lo[k] = 0xFFFFFFFFu;
-          if (e < total) {
-            // largest i >= from with off[i] <= e (owners are monotone in k)
-            uint32_t l = from, h = nready;
-            while (h - l > 1) {
-              const uint32_t mid = (l + h) >> 1;
-              if (s.off[mid] <= e) l = mid; else h = mid;
-            }
-            lo[k] = l;
-            from = l;
+          const uint32_t e = e0 + k;
+          val[k] = e < total;
+          if (val[k]) {
+            while (o < ohi && s.off[o + 1] <= e) ++o;
+            own[k] = o;
+            const uint32_t ce = s.start[o] + (e - s.off[o]);
+            w[k] = app.neighbor(ce);
+            if (P.dbg_edge) atomicAdd(P.dbg_edge + ce, 1u);
           }
         }
 #pragma unroll
         for (int k = 0; k < kU; ++k)
-          if (lo[k] != 0xFFFFFFFFu) {
-            const uint32_t e = s.start[lo[k]] + (base + k * G + r - s.off[lo[k]]);
-            w[k] = app.neighbor(e);
-            if (P.dbg_edge) atomicAdd(P.dbg_edge + e, 1u);
-          }
-#pragma unroll
-        for (int k = 0; k < kU; ++k)
-          if (lo[k] != 0xFFFFFFFFu) tk[k] = app.pre(s.pay[lo[k]], w[k]);
+          if (val[k]) tk[k] = app.pre(s.pay[own[k]], w[k]);
+        bool want[kU];
+        uint32_t out[kU];
 #pragma unroll
         for (int k = 0; k < kU; ++k) {
-          bool want = false;
-          uint32_t out = 0;
-          if (lo[k] != 0xFFFFFFFFu) want = app.post(s.pay[lo[k]], w[k], tk[k], out);
-          pusher.push(q, want, out, P.watchdog_ns);
+          want[k] = false;
+          out[k] = 0;
+          if (val[k]) want[k] = app.post(s.pay[own[k]], w[k], tk[k], out[k]);
         }
+        pusher.push_n<kU>(q, want, out, P.watchdog_ns);
       }
     } else if (MODE == MODE_WARP) {
       for (uint32_t k = 0; k < nready; ++k) {
@@ -577,24 +600,27 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
         const Payload p = s.pay[k];
         my_edges += (r == 0) ? dg : 0;
         for (uint32_t j = 0; j < dg; j += 32 * kU) {
+          const uint32_t j0 = j + r * kU;  // kU consecutive edges per lane
           uint32_t w[kU];
           typename App::Token tk[kU];
 #pragma unroll
           for (int k = 0; k < kU; ++k)
-            if (j + k * 32 + r < dg) {
-              w[k] = app.neighbor(st + j + k * 32 + r);
-              if (P.dbg_edge) atomicAdd(P.dbg_edge + st + j + k * 32 + r, 1u);
+            if (j0 + k < dg) {
+              w[k] = app.neighbor(st + j0 + k);
+              if (P.dbg_edge) atomicAdd(P.dbg_edge + st + j0 + k, 1u);
             }
 #pragma unroll
           for (int k = 0; k < kU; ++k)
-            if (j + k * 32 + r < dg) tk[k] = app.pre(p, w[k]);
+            if (j0 + k < dg) tk[k] = app.pre(p, w[k]);
+          bool want[kU];
+          uint32_t out[kU];
 #pragma unroll
           for (int k = 0; k < kU; ++k) {
-            bool want = false;
-            uint32_t out = 0;
-            if (j + k * 32 + r < dg) want = app.post(p, w[k], tk[k], out);
-            pusher.push(q, want, out, P.watchdog_ns);
+            want[k] = false;
+            out[k] = 0;
+            if (j0 + k < dg) want[k] = app.post(p, w[k], tk[k], out[k]);
           }
+          pusher.push_n<kU>(q, want, out, P.watchdog_ns);
         }
       }
     } else {
@@ -633,7 +659,7 @@ inline size_t relax_worker_smem(int mode, uint32_t block, uint32_t fetch) {
   uint32_t nwarps = block / 32;
   uint32_t K = mode == MODE_THREAD ? 32u * fetch : fetch;
   uint32_t groups = mode == MODE_CTA ? 1u : nwarps;
-  return (size_t)nwarps * 64 * 4 + group_smem_bytes<Payload>(K) * groups;
+  return (size_t)nwarps * kPushBuf * 4 + group_smem_bytes<Payload>(K) * groups;
 }
 
 }  // namespace atos

@@ -100,8 +100,8 @@ __global__ void k_pr_init_edges(const uint32_t* __restrict__ row_ptr, const uint
 
 // Initial frontier (R-PR-7): every vertex with residue > eps, warp-aggregated pushes.
 __global__ void k_pr_seed(const double* res, int64_t n, double eps, Ring q, unsigned long long wd) {
-  __shared__ uint32_t bufs[32 * 64];
-  WarpPusher pusher{bufs + warp_id() * 64, 0, 0};
+  __shared__ uint32_t bufs[32 * kPushBuf];
+  WarpPusher pusher = make_pusher(bufs);
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
     const int64_t v = base + threadIdx.x;
@@ -129,9 +129,9 @@ __global__ void k_pr_finalize(double* rank, const double* res, int64_t n, double
 // residue > eps.  (The sweep variant drives activation; see pagerank_single.)
 __global__ void k_pr_sweep(const double* res, int64_t n, double eps, Ring q, uint32_t check_size,
                            unsigned long long wd) {
-  __shared__ uint32_t bufs[32 * 64];
+  __shared__ uint32_t bufs[32 * kPushBuf];
   __shared__ unsigned long long s_c;
-  WarpPusher pusher{bufs + warp_id() * 64, 0, 0};
+  WarpPusher pusher = make_pusher(bufs);
   // each CTA sweeps chunks until the cursor passed n ids since kernel start
   while (true) {
     if (threadIdx.x == 0) s_c = atomicAdd(&q.ctl->check.v, (unsigned long long)check_size);
