@@ -215,10 +215,10 @@ def run_atos(args, ws, rank, local):
         obj = [uid]
         dist.broadcast_object_list(obj, src=0)
         comm = atos.Comm(ws, rank, obj[0], local)
-        vb, ve = atos.partition_range(g.n, ws, rank)
-        rp = g.row_ptr[vb:ve + 1] - g.row_ptr[vb]
-        ci = g.col[int(g.row_ptr[vb]):int(g.row_ptr[ve])]
-        csr = comm.partition(g.n, vb, ve, rp.contiguous(), ci.contiguous())
+        from paper_conf_icpp_chenbpbyo22_b200 import dist_host
+        vb, ve = dist_host.block_range(g.n, ws, rank)
+        rp, ci = dist_host.local_rows(g.row_ptr, g.col, vb, ve)
+        csr = comm.partition(g.n, vb, ve, rp, ci)
     # per-source reached vertices / edges (global) for GTEPS and algorithmic bytes
     out = torch.empty(csr.n_local if ws > 1 else g.n, dtype=torch.int32, device=dev)
     src_info = []

@@ -312,6 +312,31 @@ static int upload_part(Part& p, int64_t n_global, const int64_t* row_ptr, const 
   return ATOS_OK;
 }
 
+// Upload a partition given its LOCAL arrays: row_ptr[0..nl] (any base offset,
+// host or device) and the matching col[0..ml) (global ids).
+int upload_part_local(Part& p, const int64_t* row_ptr, const int32_t* col, int where, int64_t nl, int64_t ml) {
+  p.n_local = nl;
+  p.m_local = ml;
+  ATOS_CUDA(cudaMalloc(&p.row_ptr, (size_t)(nl + 1) * 4));
+  ATOS_CUDA(cudaMalloc(&p.col, (size_t)std::max<int64_t>(ml, 1) * 4));
+  if (where == ATOS_MEM_HOST) {
+    const int64_t base = row_ptr[0];
+    std::vector<uint32_t> rp((size_t)nl + 1);
+    for (int64_t i = 0; i <= nl; ++i) rp[(size_t)i] = (uint32_t)(row_ptr[i] - base);
+    ATOS_CUDA(cudaMemcpy(p.row_ptr, rp.data(), rp.size() * 4, cudaMemcpyHostToDevice));
+    if (ml) ATOS_CUDA(cudaMemcpy(p.col, col, (size_t)ml * 4, cudaMemcpyHostToDevice));
+    return ATOS_OK;
+  }
+  int64_t base = 0;
+  ATOS_CUDA(cudaMemcpy(&base, row_ptr, 8, cudaMemcpyDeviceToHost));
+  k_rebase_row_ptr<<<1024, 256>>>(row_ptr, p.row_ptr, nl + 1, base);
+  g_launches++;
+  ATOS_CUDA(cudaGetLastError());
+  if (ml) ATOS_CUDA(cudaMemcpy(p.col, col, (size_t)ml * 4, cudaMemcpyDeviceToDevice));
+  ATOS_CUDA(cudaDeviceSynchronize());
+  return ATOS_OK;
+}
+
 static int validate_host_csr(int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col) {
   if (row_ptr[0] != 0 || row_ptr[n] != m) {
     set_error("row_ptr[0] must be 0 and row_ptr[n] must equal m");
@@ -363,7 +388,7 @@ void destroy_part(Part& p) {
   p.row_ptr = nullptr;
   p.col = nullptr;
   DevBuf* bufs[] = {&p.ring, &p.ctl, &p.big, &p.bitmap, &p.shadow, &p.vbuf_a, &p.vbuf_b, &p.vbuf_c, &p.scratch,
-                    &p.ghost_a, &p.ghost_b, &p.touched, &p.outbox, &p.inbox};
+                    &p.ghost_a, &p.ghost_b, &p.touched, &p.outbox, &p.inbox, &p.out_val, &p.in_val, &p.pack};
   for (DevBuf* b : bufs) b->release();
   if (p.host_pinned) cudaFreeHost(p.host_pinned);
   p.host_pinned = nullptr;

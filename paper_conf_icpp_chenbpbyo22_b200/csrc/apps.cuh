@@ -27,6 +27,22 @@ namespace atos {
 constexpr uint32_t kInq = 0x80000000u;
 constexpr uint32_t kDepthMask = 0x7FFFFFFFu;
 
+// Partition view (S10).  Queue items, row_ptr and the
+// per-vertex state are LOCAL (id - vb); col holds GLOBAL ids.  A neighbour
+// outside [vb, vb+nl) is combined into the n-sized ghost array (min for BFS,
+// sum for PageRank) and listed once per round in `touched`, to be shipped to
+// its owner by the exchange.  ghost == nullptr: single partition, all local.
+struct GhostView {
+  uint32_t vb, nl;
+  void* ghost;
+  uint32_t* touched;
+  unsigned long long* ntouched;
+  __device__ __forceinline__ bool remote(uint32_t w) const { return ghost != nullptr && (w - vb) >= nl; }
+  __device__ __forceinline__ void touch(uint32_t w) const {
+    touched[atomicAdd(ntouched, 1ull)] = w;
+  }
+};
+
 struct BfsApp {
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
@@ -36,6 +52,7 @@ struct BfsApp {
   int dedupe;         // 0 -> paper-literal push on every improvement (atomicMin)
   uint8_t* shadow;    // nullptr -> prefilter on depth[] itself
   unsigned long long pol_first, pol_last;
+  GhostView gv;
 
   __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
   __device__ __forceinline__ void prepare() {
@@ -54,19 +71,25 @@ struct BfsApp {
     return deg != 0;
   }
 
-  __device__ __forceinline__ Token pre(const Payload nd, uint32_t w) const {
-    if (shadow) return ld_u8_hint(shadow + w, pol_last);
+  __device__ __forceinline__ Token pre_local(uint32_t lw) const {
+    if (shadow) return ld_u8_hint(shadow + lw, pol_last);
     uint32_t cur;
-    asm volatile("ld.global.u32 %0, [%1];" : "=r"(cur) : "l"(depth + w));
+    asm volatile("ld.global.u32 %0, [%1];" : "=r"(cur) : "l"(depth + lw));
     return cur;
   }
 
-  __device__ __forceinline__ bool post(const Payload nd, uint32_t w, Token tok, uint32_t& out) const {
+  __device__ __forceinline__ Token pre(const Payload nd, uint32_t w) const {
+    if (gv.remote(w)) return 0u;
+    return pre_local(w - gv.vb);
+  }
+
+  // relax local vertex lw with candidate depth nd; true -> enqueue lw
+  __device__ __forceinline__ bool relax_local(const Payload nd, uint32_t lw, Token tok, uint32_t& out) const {
     uint32_t expect = 0xFFFFFFFFu;  // guess: unvisited
     if (shadow) {
       if (tok != 255u && tok <= nd) return false;
       if (nd >= 255u) {  // shadow carries no information at this depth: prefilter on the word
-        asm volatile("ld.global.u32 %0, [%1];" : "=r"(expect) : "l"(depth + w));
+        asm volatile("ld.global.u32 %0, [%1];" : "=r"(expect) : "l"(depth + lw));
         if (expect != 0xFFFFFFFFu && (expect & kDepthMask) <= nd) return false;
       }
     } else {
@@ -76,7 +99,7 @@ struct BfsApp {
     bool pushed;
     if (dedupe) {
       while (true) {
-        const uint32_t old = atomicCAS(depth + w, expect, nd | kInq);
+        const uint32_t old = atomicCAS(depth + lw, expect, nd | kInq);
         if (old == expect) {
           pushed = (old == 0xFFFFFFFFu) || !(old & kInq);
           break;
@@ -85,16 +108,31 @@ struct BfsApp {
         expect = old;
       }
     } else {
-      if (atomicMin(depth + w, nd) <= nd) return false;
+      if (atomicMin(depth + lw, nd) <= nd) return false;
       pushed = true;
     }
-    if (shadow) st_u8_hint(shadow + w, nd < 255u ? nd : 255u, pol_last);
-    out = w;
+    if (shadow) st_u8_hint(shadow + lw, nd < 255u ? nd : 255u, pol_last);
+    out = lw;
     return pushed;
+  }
+
+  __device__ __forceinline__ bool post(const Payload nd, uint32_t w, Token tok, uint32_t& out) const {
+    if (gv.remote(w)) {
+      // remote relaxation: min-combine into the ghost, list it on first touch this round
+      uint32_t* g = (uint32_t*)gv.ghost + w;
+      if (ld_relaxed(g) <= nd) return false;
+      if (atomicMin(g, nd) == 0xFFFFFFFFu) gv.touch(w);
+      return false;
+    }
+    return relax_local(nd, w - gv.vb, tok, out);
   }
 
   __device__ __forceinline__ bool relax(const Payload nd, uint32_t w, uint32_t& out) const {
     return post(nd, w, pre(nd, w), out);
+  }
+  // an inbound (owner-local) relaxation from the exchange
+  __device__ __forceinline__ bool apply(const Payload nd, uint32_t lw, uint32_t& out) const {
+    return relax_local(nd, lw, pre_local(lw), out);
   }
 };
 
@@ -107,16 +145,19 @@ struct BfsApp {
 // atomic), which keeps "residue[v] > eps  =>  v queued or in flight".
 struct PrApp {
   using Payload = double;  // delta = alpha * rho / deg(v)
+  using Token = double;    // residue before our atomicAdd
   const uint32_t* __restrict__ row_ptr;
   const uint32_t* __restrict__ col;
   unsigned long long pol_first;
-  __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
-  __device__ __forceinline__ void prepare() { pol_first = policy_evict_first(); }
   double* rank;
   double* res;
   double alpha, eps;
-  int activate;  // 1: crossing activation (default); 0: sweep-only (Check_Size variant)
+  int activate;          // 1: crossing activation (default); 0: sweep-only (Check_Size variant)
   uint32_t* dbg_expand;  // debug: per-vertex count of expanding pops
+  GhostView gv;
+
+  __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
+  __device__ __forceinline__ void prepare() { pol_first = policy_evict_first(); }
 
   __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
     const double rho = __longlong_as_double(
@@ -130,17 +171,30 @@ struct PrApp {
     return true;
   }
 
-  using Token = double;  // residue before our atomicAdd
-  __device__ __forceinline__ Token pre(const Payload delta, uint32_t w) const { return atomicAdd(res + w, delta); }
-  __device__ __forceinline__ bool post(const Payload delta, uint32_t w, Token old, uint32_t& out) const {
+  __device__ __forceinline__ Token pre(const Payload delta, uint32_t w) const {
+    if (gv.remote(w)) return 0.0;
+    return atomicAdd(res + (w - gv.vb), delta);
+  }
+  __device__ __forceinline__ bool crossing(const Payload delta, uint32_t lw, Token old, uint32_t& out) const {
     if (activate && old <= eps && old + delta > eps) {
-      out = w;
+      out = lw;
       return true;
     }
     return false;
   }
+  __device__ __forceinline__ bool post(const Payload delta, uint32_t w, Token old, uint32_t& out) const {
+    if (gv.remote(w)) {
+      // remote mass: sum into the ghost, list it on first touch this round (delta > 0)
+      if (atomicAdd((double*)gv.ghost + w, delta) == 0.0) gv.touch(w);
+      return false;
+    }
+    return crossing(delta, w - gv.vb, old, out);
+  }
   __device__ __forceinline__ bool relax(const Payload delta, uint32_t w, uint32_t& out) const {
     return post(delta, w, pre(delta, w), out);
+  }
+  __device__ __forceinline__ bool apply(const Payload delta, uint32_t lw, uint32_t& out) const {
+    return crossing(delta, lw, atomicAdd(res + lw, delta), out);
   }
 };
 

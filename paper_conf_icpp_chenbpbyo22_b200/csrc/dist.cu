@@ -1,38 +1,305 @@
-// dist.cu -- partitioned BFS / PageRank (loopback partitions on one device,
-// or one partition per process over NCCL).  Filled in below.
+// dist.cu -- partition construction and the exchange layer of the
+// partitioned BFS / PageRank path (S10):
+//   * loopback: P partitions of one graph on one device in one process; the
+//     exchange is device-to-device copies (tests the whole protocol on 1 GPU);
+//   * NCCL: one partition per process (torchrun), grouped ncclSend/ncclRecv
+//     for the per-destination counts and payloads, ncclAllReduce for the
+//     global termination test.  NCCL is resolved with dlopen("libnccl.so.2")
+//     at first use, so the library carries no link-time NCCL dependency.
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+#include <mutex>
+#include <vector>
+
 #include "internal.h"
 
 namespace atos {
 
+int upload_part_local(Part& p, const int64_t* row_ptr, const int32_t* col, int where, int64_t nl, int64_t ml);
+
+// ------------------------------------------------------------ NCCL (dlopen)
+namespace {
+struct NcclApi {
+  bool ok = false;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+NcclApi& nccl() {
+  static NcclApi api;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return;
+#define SYM(f) api.f = (decltype(api.f))dlsym(h, "nccl" #f)
+    SYM(GetUniqueId);
+    SYM(CommInitRank);
+    SYM(CommDestroy);
+    SYM(Send);
+    SYM(Recv);
+    SYM(GroupStart);
+    SYM(GroupEnd);
+    SYM(AllReduce);
+    SYM(GetErrorString);
+#undef SYM
+    api.ok = api.GetUniqueId && api.CommInitRank && api.CommDestroy && api.Send && api.Recv && api.GroupStart &&
+             api.GroupEnd && api.AllReduce && api.GetErrorString;
+  });
+  return api;
+}
+}  // namespace
+
+#define ATOS_NCCL(call)                                                                        \
+  do {                                                                                        \
+    ncclResult_t e_ = (call);                                                                 \
+    if (e_ != ncclSuccess) {                                                                  \
+      set_error("%s failed: %s (%s:%d)", #call, nccl().GetErrorString(e_), __FILE__, __LINE__); \
+      return ATOS_ERR_NCCL;                                                                   \
+    }                                                                                         \
+  } while (0)
+
+// --------------------------------------------------------------- exchanges
+int exchange_loopback(std::vector<ExchangeIO>& io, size_t val_bytes, cudaStream_t s) {
+  const size_t P = io.size();
+  for (size_t d = 0; d < P; ++d) {
+    uint64_t total = 0;
+    for (size_t src = 0; src < P; ++src) total += io[src].counts[d];
+    io[d].in_total = total;
+    ATOS_TRY(io[d].in_vid->ensure(std::max<uint64_t>(total, 1) * 4));
+    ATOS_TRY(io[d].in_val->ensure(std::max<uint64_t>(total, 1) * val_bytes));
+  }
+  for (size_t src = 0; src < P; ++src) {
+    uint64_t seg = 0;
+    for (size_t d = 0; d < P; ++d) {
+      const uint64_t c = io[src].counts[d];
+      if (c) {
+        // offset of src's segment inside d's inbox
+        uint64_t off = 0;
+        for (size_t s2 = 0; s2 < src; ++s2) off += io[s2].counts[d];
+        ATOS_CUDA(cudaMemcpyAsync(io[d].in_vid->as<uint32_t>() + off, io[src].out_vid + seg, c * 4,
+                                  cudaMemcpyDeviceToDevice, s));
+        ATOS_CUDA(cudaMemcpyAsync((char*)io[d].in_val->p + off * val_bytes,
+                                  (const char*)io[src].out_val + seg * val_bytes, c * val_bytes,
+                                  cudaMemcpyDeviceToDevice, s));
+      }
+      seg += c;
+    }
+  }
+  return ATOS_OK;
+}
+
+int exchange_nccl(Comm* c, ExchangeIO& io, size_t val_bytes, cudaStream_t s, uint64_t* bytes_sent) {
+  NcclApi& api = nccl();
+  const int P = c->nranks;
+  ncclComm_t comm = (ncclComm_t)c->nccl;
+  // 1. counts: P u64 out, P u64 in (device staging in the inbox buffers' scratch)
+  static thread_local DevBuf cbuf;
+  ATOS_TRY(cbuf.ensure(sizeof(uint64_t) * 2 * P));
+  uint64_t* d_send = cbuf.as<uint64_t>();
+  uint64_t* d_recv = d_send + P;
+  ATOS_CUDA(cudaMemcpyAsync(d_send, io.counts.data(), sizeof(uint64_t) * P, cudaMemcpyHostToDevice, s));
+  ATOS_NCCL(api.GroupStart());
+  for (int p = 0; p < P; ++p) {
+    ATOS_NCCL(api.Send(d_send + p, 1, ncclUint64, p, comm, s));
+    ATOS_NCCL(api.Recv(d_recv + p, 1, ncclUint64, p, comm, s));
+  }
+  ATOS_NCCL(api.GroupEnd());
+  std::vector<uint64_t> rc(P);
+  ATOS_CUDA(cudaMemcpyAsync(rc.data(), d_recv, sizeof(uint64_t) * P, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  uint64_t total = 0;
+  for (int p = 0; p < P; ++p) total += rc[p];
+  io.in_total = total;
+  ATOS_TRY(io.in_vid->ensure(std::max<uint64_t>(total, 1) * 4));
+  ATOS_TRY(io.in_val->ensure(std::max<uint64_t>(total, 1) * val_bytes));
+  // 2. payloads (SoA: ids then values), one grouped round of sends/recvs
+  ATOS_NCCL(api.GroupStart());
+  uint64_t so = 0, ro = 0, b = 0;
+  for (int p = 0; p < P; ++p) {
+    if (io.counts[p]) {
+      ATOS_NCCL(api.Send(io.out_vid + so, io.counts[p], ncclUint32, p, comm, s));
+      ATOS_NCCL(api.Send((const char*)io.out_val + so * val_bytes, io.counts[p] * val_bytes, ncclUint8, p, comm, s));
+      if (p != c->rank) b += io.counts[p] * (4 + val_bytes);
+    }
+    if (rc[p]) {
+      ATOS_NCCL(api.Recv(io.in_vid->as<uint32_t>() + ro, rc[p], ncclUint32, p, comm, s));
+      ATOS_NCCL(api.Recv((char*)io.in_val->p + ro * val_bytes, rc[p] * val_bytes, ncclUint8, p, comm, s));
+    }
+    so += io.counts[p];
+    ro += rc[p];
+  }
+  ATOS_NCCL(api.GroupEnd());
+  if (bytes_sent) *bytes_sent = b;
+  return ATOS_OK;
+}
+
+int allreduce_u64(Comm* c, uint64_t* v, cudaStream_t s) {
+  static thread_local DevBuf buf;
+  ATOS_TRY(buf.ensure(8));
+  ATOS_CUDA(cudaMemcpyAsync(buf.p, v, 8, cudaMemcpyHostToDevice, s));
+  ATOS_NCCL(nccl().AllReduce(buf.p, buf.p, 1, ncclUint64, ncclSum, (ncclComm_t)c->nccl, s));
+  ATOS_CUDA(cudaMemcpyAsync(v, buf.p, 8, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  return ATOS_OK;
+}
+
+int allreduce_f64(Comm* c, double* v, cudaStream_t s) {
+  static thread_local DevBuf buf;
+  ATOS_TRY(buf.ensure(8));
+  ATOS_CUDA(cudaMemcpyAsync(buf.p, v, 8, cudaMemcpyHostToDevice, s));
+  ATOS_NCCL(nccl().AllReduce(buf.p, buf.p, 1, ncclFloat64, ncclSum, (ncclComm_t)c->nccl, s));
+  ATOS_CUDA(cudaMemcpyAsync(v, buf.p, 8, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  return ATOS_OK;
+}
+
+// ----------------------------------------------------- partition creation
 int create_loopback_parts(atos_csr* g, const int64_t* row_ptr, const int32_t* col, int where) {
-  set_error("partitioned graphs not built yet");
-  return ATOS_ERR_UNSUPPORTED;
-}
-int bfs_partitioned(atos_csr* g, int64_t src, uint32_t* depth_dev, const Resolved& r, atos_stats* st) {
-  set_error("partitioned BFS not built yet");
-  return ATOS_ERR_UNSUPPORTED;
-}
-int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_dev, const Resolved& r,
-                         atos_stats* st) {
-  set_error("partitioned PageRank not built yet");
-  return ATOS_ERR_UNSUPPORTED;
+  const int P = g->num_parts;
+  g->parts.resize(P);
+  for (int p = 0; p < P; ++p) {
+    int64_t vb = 0, ve = 0;
+    atos_partition_range(g->n, P, p, &vb, &ve);
+    int64_t eb = 0, ee = 0;
+    if (where == ATOS_MEM_HOST) {
+      eb = row_ptr[vb];
+      ee = row_ptr[ve];
+    } else {
+      ATOS_CUDA(cudaMemcpy(&eb, row_ptr + vb, 8, cudaMemcpyDeviceToHost));
+      ATOS_CUDA(cudaMemcpy(&ee, row_ptr + ve, 8, cudaMemcpyDeviceToHost));
+    }
+    Part& part = g->parts[p];
+    ATOS_TRY(upload_part_local(part, row_ptr + vb, col + eb, where, ve - vb, ee - eb));
+    // rebase: upload_part_local expects offsets relative to row_ptr[vb]
+    part.v_begin = vb;
+    part.v_end = ve;
+  }
+  return ATOS_OK;
 }
 
 }  // namespace atos
 
+using namespace atos;
+
+struct atos_comm {
+  Comm c;
+};
+
 extern "C" {
+
 int atos_comm_unique_id(void* id_out, size_t len) {
-  atos::set_error("NCCL communicator not built yet");
-  return ATOS_ERR_UNSUPPORTED;
+  if (!id_out || len < sizeof(ncclUniqueId)) {
+    set_error("atos_comm_unique_id: need a buffer of %zu bytes", sizeof(ncclUniqueId));
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (!nccl().ok) {
+    set_error("atos_comm_unique_id: libnccl.so.2 could not be loaded");
+    return ATOS_ERR_NCCL;
+  }
+  ncclUniqueId id;
+  ATOS_NCCL(nccl().GetUniqueId(&id));
+  memcpy(id_out, &id, sizeof(id));
+  return ATOS_OK;
 }
+
 int atos_comm_create(atos_comm** out, int nranks, int rank, const void* id, size_t len, int device) {
-  atos::set_error("NCCL communicator not built yet");
-  return ATOS_ERR_UNSUPPORTED;
+  if (!out || nranks < 1 || rank < 0 || rank >= nranks || !id || len < sizeof(ncclUniqueId)) {
+    set_error("atos_comm_create: invalid argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  *out = nullptr;
+  if (!nccl().ok) {
+    set_error("atos_comm_create: libnccl.so.2 could not be loaded");
+    return ATOS_ERR_NCCL;
+  }
+  DeviceGuard dg(device);
+  ncclUniqueId uid;
+  memcpy(&uid, id, sizeof(uid));
+  ncclComm_t comm = nullptr;
+  ATOS_NCCL(nccl().CommInitRank(&comm, nranks, uid, rank));
+  atos_comm* c = new atos_comm();
+  c->c.nranks = nranks;
+  c->c.rank = rank;
+  c->c.device = device;
+  c->c.nccl = comm;
+  *out = c;
+  return ATOS_OK;
 }
-void atos_comm_destroy(atos_comm* comm) {}
+
+void atos_comm_destroy(atos_comm* c) {
+  if (!c) return;
+  if (c->c.nccl && nccl().ok) nccl().CommDestroy((ncclComm_t)c->c.nccl);
+  delete c;
+}
+
 int atos_csr_create_part(atos_csr** out, atos_comm* comm, int64_t n_global, int64_t v_begin, int64_t v_end,
                          int64_t m_local, const int64_t* row_ptr_local, const int32_t* col_global, int where) {
-  atos::set_error("partitioned graphs not built yet");
-  return ATOS_ERR_UNSUPPORTED;
+  if (!out || !comm || n_global < 0 || v_begin < 0 || v_end < v_begin || v_end > n_global || m_local < 0 ||
+      (v_end > v_begin && !row_ptr_local) || (m_local > 0 && !col_global)) {
+    set_error("atos_csr_create_part: invalid argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  *out = nullptr;
+  int64_t eb = 0, ee = 0;
+  atos_partition_range(n_global, comm->c.nranks, comm->c.rank, &eb, &ee);
+  if (eb != v_begin || ee != v_end) {
+    set_error("atos_csr_create_part: rank %d must own [%lld, %lld) (atos_partition_range), got [%lld, %lld)",
+              comm->c.rank, (long long)eb, (long long)ee, (long long)v_begin, (long long)v_end);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (m_local >= (int64_t)0xFFFFFFFFll || n_global >= (int64_t)0x7FFFFFFFll) {
+    set_error("atos_csr_create_part: n < 2^31 and m_local < 2^32 required");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  if (where == ATOS_MEM_HOST) {
+    const int64_t nl = v_end - v_begin;
+    if (nl > 0 && (row_ptr_local[0] != 0 || row_ptr_local[nl] != m_local)) {
+      set_error("atos_csr_create_part: row_ptr_local must start at 0 and end at m_local");
+      return ATOS_ERR_INVALID_ARG;
+    }
+    for (int64_t i = 0; i < nl; ++i)
+      if (row_ptr_local[i + 1] < row_ptr_local[i]) {
+        set_error("atos_csr_create_part: row_ptr_local not non-decreasing at %lld", (long long)i);
+        return ATOS_ERR_INVALID_ARG;
+      }
+    for (int64_t e = 0; e < m_local; ++e)
+      if (col_global[e] < 0 || (int64_t)col_global[e] >= n_global) {
+        set_error("atos_csr_create_part: col_global[%lld] out of range", (long long)e);
+        return ATOS_ERR_INVALID_ARG;
+      }
+  }
+  DeviceGuard dg(comm->c.device);
+  atos_csr* g = new atos_csr();
+  g->device = comm->c.device;
+  g->n = n_global;
+  g->m = m_local;
+  g->num_parts = 1;
+  g->comm = &comm->c;
+  g->rank = comm->c.rank;
+  g->nranks = comm->c.nranks;
+  g->parts.resize(1);
+  int rc = upload_part_local(g->parts[0], row_ptr_local, col_global, where, v_end - v_begin, m_local);
+  if (rc == ATOS_OK) {
+    g->parts[0].v_begin = v_begin;
+    g->parts[0].v_end = v_end;
+  } else {
+    atos_csr_destroy(g);
+    return rc;
+  }
+  *out = g;
+  return ATOS_OK;
 }
-}
+
+}  // extern "C"

@@ -51,13 +51,33 @@ struct Part {
   uint32_t* col = nullptr;          // m_local, GLOBAL ids (single-partition: the ids)
   // cached workspaces (grow-only, reused across calls)
   DevBuf ring, ctl, big, bitmap, shadow, vbuf_a, vbuf_b, vbuf_c, scratch;
-  DevBuf ghost_a, ghost_b, touched, outbox, inbox;
+  DevBuf ghost_a, ghost_b, touched, outbox, inbox, out_val, in_val, pack;
   uint64_t ring_cap = 0;
   void* host_pinned = nullptr;      // 4 KB pinned scratch for control-block reads
   bool ring_clean = false;          // every ring slot is EMPTY
 };
 
-struct Comm;
+// Multi-process communicator (dist.cu): NCCL loaded at run time (dlopen of
+// libnccl.so.2 -- the copy torch already loaded), so the library has no link
+// dependency on NCCL and CPU-only processes never touch it.
+struct Comm {
+  int nranks = 1, rank = 0, device = 0;
+  void* nccl = nullptr;  // ncclComm_t
+};
+
+// One partition's side of an exchange round.
+struct ExchangeIO {
+  uint32_t* out_vid = nullptr;        // outbox ids (owner-local), grouped by destination part
+  void* out_val = nullptr;            // outbox values (u32 depth or f64 mass)
+  std::vector<uint64_t> counts;       // items for each destination part (P entries)
+  DevBuf* in_vid = nullptr;           // inbox (grown as needed)
+  DevBuf* in_val = nullptr;
+  uint64_t in_total = 0;
+};
+int exchange_loopback(std::vector<ExchangeIO>& io, size_t val_bytes, cudaStream_t s);
+int exchange_nccl(Comm* c, ExchangeIO& io, size_t val_bytes, cudaStream_t s, uint64_t* bytes_sent);
+int allreduce_u64(Comm* c, uint64_t* v, cudaStream_t s);
+int allreduce_f64(Comm* c, double* v, cudaStream_t s);
 
 }  // namespace atos
 

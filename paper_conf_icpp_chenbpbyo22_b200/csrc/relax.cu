@@ -112,11 +112,11 @@ __global__ void k_pr_seed(const double* res, int64_t n, double eps, Ring q, unsi
   if (lane_id() == 0) atomicAdd(&q.ctl->stat_pushes.v, (unsigned long long)pusher.total);
 }
 
-// rank_out = rank / n (R-PR-4); residual sum into *sum (conservation check).
-__global__ void k_pr_finalize(double* rank, const double* res, int64_t n, double* sum) {
+// rank_out = rank / n_global (R-PR-4); residual sum into *sum (conservation check).
+__global__ void k_pr_finalize_n(double* rank, const double* res, int64_t n, double n_global, double* sum) {
   double acc = 0.0;
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-    rank[v] = rank[v] / (double)n;
+    rank[v] = rank[v] / n_global;
     acc += res[v];
   }
   for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
@@ -290,7 +290,7 @@ int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolve
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, depth, (size_t)n * 4, true);
-  BfsApp app{p.row_ptr, p.col, depth, r.dedupe, shadow, 0ull, 0ull};
+  BfsApp app{p.row_ptr, p.col, depth, r.dedupe, shadow, 0ull, 0ull, GhostView{0u, (uint32_t)n, nullptr, nullptr, nullptr}};
   p.ring_clean = false;
   int rc = launch_relax(app, q, r, p, st);
   if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
@@ -324,7 +324,8 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, res, (size_t)n * 8, true);
-  PrApp app{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, r.check_size > 0 ? 0 : 1, nullptr};
+  PrApp app{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, r.check_size > 0 ? 0 : 1, nullptr,
+            GhostView{0u, (uint32_t)n, nullptr, nullptr, nullptr}};
   uint32_t* dbg_edge = nullptr;
   const bool dbg = getenv("ATOS_DEBUG_EDGES") != nullptr;
   if (dbg) {
@@ -392,7 +393,7 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
   }
   if (rc != ATOS_OK) return rc;
   ATOS_CUDA(cudaMemsetAsync(sum, 0, 8, s));
-  k_pr_finalize<<<gs, 256, 0, s>>>(rank, res, n, sum);
+  k_pr_finalize_n<<<gs, 256, 0, s>>>(rank, res, n, (double)n, sum);
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   rc = finish_queue(p, s, st, "pagerank");
@@ -402,6 +403,323 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
     ATOS_CUDA(cudaMemcpy(&h_sum, sum, 8, cudaMemcpyDeviceToHost));
     st->residual_sum = h_sum;
   }
+  return ATOS_OK;
+}
+
+}  // namespace atos
+
+// =========================================================================
+// Partitioned BFS / PageRank (S10): rounds of
+//   local persistent phase -> pack touched ghosts per owner -> exchange ->
+//   apply inbox (relax + activate) -> global "anything sent?" reduction.
+// Loopback (P partitions in one process) and NCCL (one partition per rank)
+// share this code; only the exchange/reduction differ.
+// =========================================================================
+namespace atos {
+
+// count touched ghosts per destination part
+__global__ void k_pack_count(const uint32_t* touched, const unsigned long long* ntouched, uint32_t chunk,
+                             unsigned long long* counts) {
+  const unsigned long long nt = *ntouched;
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < nt;
+       i += (unsigned long long)gridDim.x * blockDim.x)
+    atomicAdd(counts + touched[i] / chunk, 1ull);
+}
+
+// exclusive scan of the P counts into cursors (P is small)
+__global__ void k_pack_scan(const unsigned long long* counts, unsigned long long* cursor, uint32_t P) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    unsigned long long acc = 0;
+    for (uint32_t d = 0; d < P; ++d) {
+      cursor[d] = acc;
+      acc += counts[d];
+    }
+  }
+}
+
+// write (owner-local id, combined value) grouped by owner; reset the ghost
+template <class V>
+__global__ void k_pack_write(const uint32_t* touched, unsigned long long* ntouched, V* ghost, uint32_t chunk,
+                             unsigned long long* cursor, uint32_t* out_vid, V* out_val, V reset) {
+  const unsigned long long nt = *ntouched;
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < nt;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    const uint32_t w = touched[i], owner = w / chunk;
+    const unsigned long long pos = atomicAdd(cursor + owner, 1ull);
+    out_vid[pos] = w - owner * chunk;
+    out_val[pos] = ghost[w];
+    ghost[w] = reset;
+  }
+}
+
+__global__ void k_reset_u64(unsigned long long* p) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) *p = 0;
+}
+
+// apply an inbox: owner-local relax + activation through the normal queue
+template <class App>
+__global__ void k_apply(App app, const uint32_t* vid, const typename App::Payload* val, unsigned long long total,
+                        Ring q, unsigned long long wd) {
+  __shared__ uint32_t bufs[32 * kPushBuf];
+  WarpPusher pusher = make_pusher(bufs);
+  app.prepare();
+  const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+  for (unsigned long long base = (unsigned long long)blockIdx.x * blockDim.x; base < total; base += stride) {
+    const unsigned long long i = base + threadIdx.x;
+    bool want = false;
+    uint32_t out = 0;
+    if (i < total) want = app.apply(val[i], vid[i], out);
+    pusher.push(q, want, out, wd);
+  }
+  pusher.flush(q, wd);
+  if (lane_id() == 0) atomicAdd(&q.ctl->stat_pushes.v, (unsigned long long)pusher.total);
+}
+
+// PageRank residue init for a partition: local rows, GLOBAL columns
+__global__ void k_pr_init_edges_part(const uint32_t* __restrict__ row_ptr, const uint32_t* __restrict__ col,
+                                     double* res, uint32_t nl, uint32_t m, double c, GhostView gv) {
+  __shared__ uint32_t s_r[2];
+  for (uint64_t t0 = (uint64_t)blockIdx.x * blockDim.x; t0 < m; t0 += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t e0 = (uint32_t)t0;
+    const uint64_t tend = t0 + blockDim.x < (uint64_t)m ? t0 + blockDim.x : (uint64_t)m;
+    const uint32_t e1 = (uint32_t)(tend - 1);
+    if (threadIdx.x == 0) s_r[0] = row_of(row_ptr, 0, nl - 1, e0);
+    if (threadIdx.x == 32 || (blockDim.x <= 32 && threadIdx.x == 0)) s_r[1] = row_of(row_ptr, 0, nl - 1, e1);
+    __syncthreads();
+    const uint32_t e = e0 + threadIdx.x;
+    if (e <= e1) {
+      const uint32_t v = row_of(row_ptr, s_r[0], s_r[1], e);
+      const uint32_t deg = __ldg(row_ptr + v + 1) - __ldg(row_ptr + v);
+      const uint32_t w = __ldg(col + e);
+      const double add = c / (double)deg;
+      if (gv.remote(w)) {
+        if (atomicAdd((double*)gv.ghost + w, add) == 0.0) gv.touch(w);
+      } else {
+        red_add_f64(res + (w - gv.vb), add);
+      }
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void k_bfs_init_part(uint32_t* depth, int dedupe, uint8_t* shadow, Ring q, uint32_t lsrc, int has_src,
+                                unsigned long long wd) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    run_begin(q.ctl);
+    if (has_src) {
+      depth[lsrc] = dedupe ? kInq : 0u;
+      if (shadow) shadow[lsrc] = 0;
+      const unsigned long long idx = q.ctl->tail.v;
+      q.ctl->tail.v = idx + 1;
+      publish_one(q, idx, lsrc, wd);
+    }
+  }
+}
+
+namespace {
+
+struct PartRun {
+  Part* p;
+  uint32_t* state;      // depth (u32) or rank (f64) -- local slice of the output
+  GhostView gv;
+  unsigned long long* counts;   // device: P counts, then P cursors
+  unsigned long long* ntouched; // device
+};
+
+template <class V>
+int pack_part(PartRun& pr, uint32_t chunk, uint32_t P, V reset, ExchangeIO& io, cudaStream_t s) {
+  Part& p = *pr.p;
+  ATOS_CUDA(cudaMemsetAsync(pr.counts, 0, sizeof(unsigned long long) * P, s));
+  k_pack_count<<<592, 256, 0, s>>>(p.touched.as<uint32_t>(), pr.ntouched, chunk, pr.counts);
+  k_pack_scan<<<1, 32, 0, s>>>(pr.counts, pr.counts + P, P);
+  k_pack_write<V><<<592, 256, 0, s>>>(p.touched.as<uint32_t>(), pr.ntouched, (V*)pr.gv.ghost, chunk, pr.counts + P,
+                                      p.outbox.as<uint32_t>(), p.out_val.as<V>(), reset);
+  k_reset_u64<<<1, 32, 0, s>>>(pr.ntouched);
+  g_launches += 4;
+  ATOS_CUDA(cudaGetLastError());
+  std::vector<unsigned long long> h(P);
+  ATOS_CUDA(cudaMemcpyAsync(h.data(), pr.counts, sizeof(unsigned long long) * P, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  io.out_vid = p.outbox.as<uint32_t>();
+  io.out_val = p.out_val.p;
+  io.counts.assign(h.begin(), h.end());
+  io.in_vid = &p.inbox;
+  io.in_val = &p.in_val;
+  return ATOS_OK;
+}
+
+// allocate the ghost machinery of one partition (n_global-sized ghost, touched list, outbox)
+int ensure_ghosts(Part& p, int64_t n_global, size_t val_bytes, uint32_t P, cudaStream_t s) {
+  ATOS_TRY(p.ghost_a.ensure((size_t)n_global * val_bytes));
+  ATOS_TRY(p.touched.ensure((size_t)n_global * 4));
+  ATOS_TRY(p.outbox.ensure((size_t)n_global * 4));
+  ATOS_TRY(p.out_val.ensure((size_t)n_global * val_bytes));
+  ATOS_TRY(p.pack.ensure(sizeof(unsigned long long) * (2 * P + 2)));
+  return ATOS_OK;
+}
+
+template <class App, class V>
+int run_rounds(atos_csr* g, std::vector<PartRun>& runs, std::vector<App>& apps, const Resolved& r, V reset,
+               atos_stats* st) {
+  cudaStream_t s = r.stream;
+  const uint32_t P = g->comm ? (uint32_t)g->nranks : (uint32_t)g->num_parts;
+  const uint32_t chunk = (uint32_t)((g->n + P - 1) / P);
+  Resolved rl = r;
+  rl.persistent = 1;  // each local phase runs to local quiescence
+  uint64_t rounds = 0, bytes = 0;
+  std::vector<ExchangeIO> io(runs.size());
+  while (true) {
+    for (size_t i = 0; i < runs.size(); ++i) {
+      Part& p = *runs[i].p;
+      Ring q = ring_of(p);
+      ATOS_TRY(launch_relax(apps[i], q, rl, p, st));
+    }
+    for (size_t i = 0; i < runs.size(); ++i) ATOS_TRY(pack_part<V>(runs[i], chunk, P, reset, io[i], s));
+    uint64_t sent = 0;
+    for (auto& x : io)
+      for (uint32_t d = 0; d < P; ++d) sent += x.counts[d];
+    if (g->comm) {
+      uint64_t b = 0;
+      ATOS_TRY(exchange_nccl(g->comm, io[0], sizeof(V), s, &b));
+      bytes += b;
+      ATOS_TRY(allreduce_u64(g->comm, &sent, s));
+    } else {
+      for (auto& x : io)
+        for (uint32_t d = 0; d < P; ++d) bytes += x.counts[d] * (4 + sizeof(V));
+      ATOS_TRY(exchange_loopback(io, sizeof(V), s));
+    }
+    ++rounds;
+    if (sent == 0) break;
+    for (size_t i = 0; i < runs.size(); ++i) {
+      if (!io[i].in_total) continue;
+      Part& p = *runs[i].p;
+      Ring q = ring_of(p);
+      k_apply<App><<<(unsigned)std::min<uint64_t>((io[i].in_total + 1023) / 1024, 1184), 1024, 0, s>>>(
+          apps[i], io[i].in_vid->as<uint32_t>(), (const typename App::Payload*)io[i].in_val->p, io[i].in_total, q,
+          r.watchdog_ns);
+      ++g_launches;
+      ATOS_CUDA(cudaGetLastError());
+    }
+    if (rounds > 100000) {
+      set_error("partitioned run did not converge within 100000 rounds");
+      return ATOS_ERR_TIMEOUT;
+    }
+  }
+  for (auto& pr : runs) ATOS_TRY(finish_queue(*pr.p, s, st, "partitioned"));
+  if (st) {
+    st->rounds = rounds;
+    st->bytes_exchanged += bytes;
+  }
+  return ATOS_OK;
+}
+
+}  // namespace
+
+int bfs_partitioned(atos_csr* g, int64_t src, uint32_t* depth_out, const Resolved& r, atos_stats* st) {
+  cudaStream_t s = r.stream;
+  const uint32_t P = g->comm ? (uint32_t)g->nranks : (uint32_t)g->num_parts;
+  std::vector<PartRun> runs(g->parts.size());
+  std::vector<BfsApp> apps(g->parts.size());
+  for (size_t i = 0; i < g->parts.size(); ++i) {
+    Part& p = g->parts[i];
+    const int64_t n = p.n_local;
+    ATOS_TRY(ensure_queue(p, pow2_at_least((uint64_t)std::max<int64_t>(2 * n, 1024)), s));
+    ATOS_TRY(ensure_ghosts(p, g->n, 4, P, s));
+    ATOS_TRY(p.shadow.ensure((size_t)std::max<int64_t>(n, 1)));
+    // loopback: the partition writes its slice of the full output; NCCL: the local output
+    uint32_t* depth = g->comm ? depth_out : depth_out + p.v_begin;
+    if (n) ATOS_CUDA(cudaMemsetAsync(depth, 0xFF, (size_t)n * 4, s));
+    ATOS_CUDA(cudaMemsetAsync(p.shadow.p, 0xFF, (size_t)std::max<int64_t>(n, 1), s));
+    ATOS_CUDA(cudaMemsetAsync(p.ghost_a.p, 0xFF, (size_t)g->n * 4, s));
+    unsigned long long* pk = p.pack.as<unsigned long long>();
+    ATOS_CUDA(cudaMemsetAsync(pk, 0, sizeof(unsigned long long) * (2 * P + 2), s));
+    PartRun& pr = runs[i];
+    pr.p = &p;
+    pr.state = depth;
+    pr.counts = pk;
+    pr.ntouched = pk + 2 * P;
+    pr.gv = GhostView{(uint32_t)p.v_begin, (uint32_t)n, p.ghost_a.p, p.touched.as<uint32_t>(), pr.ntouched};
+    const bool has = src >= p.v_begin && src < p.v_end;
+    Ring q = ring_of(p);
+    k_bfs_init_part<<<1, 32, 0, s>>>(depth, r.dedupe, p.shadow.as<uint8_t>(), q,
+                                     has ? (uint32_t)(src - p.v_begin) : 0u, has ? 1 : 0, r.watchdog_ns);
+    ++g_launches;
+    p.ring_clean = false;
+    apps[i] = BfsApp{p.row_ptr, p.col, depth, r.dedupe, p.shadow.as<uint8_t>(), 0ull, 0ull, pr.gv};
+  }
+  ATOS_CUDA(cudaGetLastError());
+  return run_rounds<BfsApp, uint32_t>(g, runs, apps, r, 0xFFFFFFFFu, st);
+}
+
+int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_out, const Resolved& r,
+                         atos_stats* st) {
+  cudaStream_t s = r.stream;
+  const uint32_t P = g->comm ? (uint32_t)g->nranks : (uint32_t)g->num_parts;
+  if (r.check_size > 0) {
+    set_error("check_size sweeps are single-partition only");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  std::vector<PartRun> runs(g->parts.size());
+  std::vector<PrApp> apps(g->parts.size());
+  const int gs = 148 * 8;
+  for (size_t i = 0; i < g->parts.size(); ++i) {
+    Part& p = g->parts[i];
+    const int64_t n = p.n_local;
+    ATOS_TRY(ensure_queue(p, pow2_at_least((uint64_t)std::max<int64_t>(2 * n, 1024)), s));
+    ATOS_TRY(ensure_ghosts(p, g->n, 8, P, s));
+    ATOS_TRY(p.vbuf_a.ensure((size_t)std::max<int64_t>(n, 1) * 8));
+    double* rank = g->comm ? rank_out : rank_out + p.v_begin;
+    double* res = p.vbuf_a.as<double>();
+    ATOS_CUDA(cudaMemsetAsync(p.ghost_a.p, 0, (size_t)g->n * 8, s));
+    unsigned long long* pk = p.pack.as<unsigned long long>();
+    ATOS_CUDA(cudaMemsetAsync(pk, 0, sizeof(unsigned long long) * (2 * P + 2), s));
+    PartRun& pr = runs[i];
+    pr.p = &p;
+    pr.state = nullptr;
+    pr.counts = pk;
+    pr.ntouched = pk + 2 * P;
+    pr.gv = GhostView{(uint32_t)p.v_begin, (uint32_t)n, p.ghost_a.p, p.touched.as<uint32_t>(), pr.ntouched};
+    Ring q = ring_of(p);
+    k_run_begin<<<1, 32, 0, s>>>(q.ctl);
+    if (n) {
+      k_pr_init_vertices<<<gs, 256, 0, s>>>(rank, res, n, 1.0 - alpha);
+      g_launches += 1;
+    }
+    if (p.m_local) {
+      k_pr_init_edges_part<<<gs * 2, 256, 0, s>>>(p.row_ptr, p.col, res, (uint32_t)n, (uint32_t)p.m_local,
+                                                  (1.0 - alpha) * alpha, pr.gv);
+      ++g_launches;
+    }
+    if (n) {
+      k_pr_seed<<<gs, 1024, 0, s>>>(res, n, eps, q, r.watchdog_ns);
+      ++g_launches;
+    }
+    g_launches += 1;
+    p.ring_clean = false;
+    apps[i] = PrApp{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, 1, nullptr, pr.gv};
+  }
+  ATOS_CUDA(cudaGetLastError());
+  ATOS_TRY((run_rounds<PrApp, double>(g, runs, apps, r, 0.0, st)));
+  // finalize: rank / n_global, residual sum over all partitions (conservation)
+  double total = 0.0;
+  for (size_t i = 0; i < g->parts.size(); ++i) {
+    Part& p = g->parts[i];
+    ATOS_TRY(p.scratch.ensure(64));
+    double* sum = p.scratch.as<double>();
+    ATOS_CUDA(cudaMemsetAsync(sum, 0, 8, s));
+    double* rank = g->comm ? rank_out : rank_out + p.v_begin;
+    if (p.n_local) {
+      // rank_out = rank / n_global
+      k_pr_finalize_n<<<gs, 256, 0, s>>>(rank, p.vbuf_a.as<double>(), p.n_local, (double)g->n, sum);
+      ++g_launches;
+    }
+    double h = 0;
+    ATOS_CUDA(cudaMemcpyAsync(&h, sum, 8, cudaMemcpyDeviceToHost, s));
+    ATOS_CUDA(cudaStreamSynchronize(s));
+    total += h;
+  }
+  if (g->comm) ATOS_TRY(allreduce_f64(g->comm, &total, s));
+  if (st) st->residual_sum = total;
   return ATOS_OK;
 }
 

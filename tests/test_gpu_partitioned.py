@@ -1,0 +1,106 @@
+"""GPU: the partitioned (multi-GPU) BFS / PageRank protocol of S10 run with P
+loopback partitions on one device -- same rounds, ghost combining, packing,
+exchange and apply as the NCCL path, exchange by device copies.  BFS must stay
+bit-exact and PageRank within the north_star tolerance + conservation (ghost
+mass must never be lost)."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_icpp_chenbpbyo22_b200 as atos
+from paper_conf_icpp_chenbpbyo22_b200 import gen
+
+import _graphs as G
+from _gpu import DEV, as_u32, check_pr, csr_of
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def rmat13():
+    g = gen.rmat(13, 16, seed=21)
+    rp, ci = g.numpy()
+    return g, rp, ci
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+@pytest.mark.parametrize("knobs", [dict(), dict(worker=32, fetch_size=8), dict(dedupe=0)], ids=["cta", "warp", "nodedupe"])
+def test_bfs_loopback_rmat(rmat13, P, knobs):
+    g, rp, ci = rmat13
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=P)
+    for s in (gen.pick_source(g, 1), 0, g.n - 1):
+        d, st = atos.bfs(csr, s, **knobs)
+        np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, s))
+        assert st["rounds"] >= 1
+
+
+@pytest.mark.parametrize("P", [2, 5])
+def test_bfs_loopback_mesh(P):
+    R, C = 120, 97
+    g = gen.mesh(R, C)
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=P)
+    r, c = np.divmod(np.arange(R * C), C)
+    for (r0, c0) in ((0, 0), (R // 2, C // 2)):
+        d, st = atos.bfs(csr, r0 * C + c0)
+        np.testing.assert_array_equal(as_u32(d), np.abs(r - r0) + np.abs(c - c0))
+
+
+def test_bfs_loopback_directed_and_host_output():
+    import torch
+    rp, ci = G.csr_from_edges(7, [(0, 1), (1, 2), (2, 3), (3, 4), (4, 5), (5, 6), (6, 0)])
+    csr = csr_of(rp, ci, num_parts=3)
+    out = torch.empty(7, dtype=torch.int32)
+    d, st = atos.bfs(csr, 4, out=out)
+    np.testing.assert_array_equal(d.numpy().view(np.uint32), oracle.bfs(rp, ci, 4))
+
+
+@pytest.mark.parametrize("P", [2, 4, 7])
+def test_pagerank_loopback_rmat(rmat13, P):
+    g, rp, ci = rmat13
+    ref, _, _ = oracle.pagerank_jacobi(rp, ci, 0.85)
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=P)
+    for knobs in (dict(), dict(worker=32, fetch_size=4)):
+        r, st = atos.pagerank(csr, 0.85, 1e-6, **knobs)
+        err = check_pr(rp, ci, r, st, 1e-6, ref=ref)
+        assert abs(err) < 1e-9 * g.n, "ghost mass lost or duplicated"
+        assert st["bytes_exchanged"] > 0
+
+
+def test_pagerank_loopback_star():
+    n = 5001
+    rp, ci = G.star(n)
+    csr = csr_of(rp, ci, num_parts=4)
+    r, st = atos.pagerank(csr, 0.85, 1e-10)
+    a = 0.85
+    xc = (1 + a * (n - 1)) / (1 + a)
+    xl = (1 - a) + a * xc / (n - 1)
+    x = r.cpu().numpy() * n
+    np.testing.assert_allclose(x[0], xc, rtol=1e-8)
+    np.testing.assert_allclose(x[1:], xl, rtol=1e-8)
+
+
+def test_color_partitioned_unsupported(rmat13):
+    g, rp, ci = rmat13
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=2)
+    with pytest.raises(RuntimeError, match="UNSUPPORTED"):
+        atos.color(csr, 1)
+
+
+def test_nccl_single_rank_communicator(rmat13):
+    """The NCCL path end to end with one rank (self send/recv + allreduce): dlopen,
+    unique id, communicator, partition creation, exchange rounds."""
+    g, rp, ci = rmat13
+    uid = atos.Comm.unique_id()
+    assert len(uid) == 128
+    comm = atos.Comm(1, 0, uid, 0)
+    vb, ve = atos.partition_range(g.n, 1, 0)
+    part = comm.partition(g.n, vb, ve, g.row_ptr.to(DEV), g.col.to(DEV))
+    s = gen.pick_source(g, 1)
+    d, st = atos.bfs(part, s)
+    np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, s))
+    r, st = atos.pagerank(part, 0.85, 1e-6)
+    check_pr(rp, ci, r, st, 1e-6)
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        comm.partition(g.n, 0, g.n - 1, g.row_ptr[:-1].to(DEV), g.col.to(DEV))
+    part.close()
+    comm.close()
