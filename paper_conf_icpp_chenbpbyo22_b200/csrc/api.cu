@@ -297,10 +297,16 @@ static int upload_part(Part& p, int64_t n_global, const int64_t* row_ptr, const 
   ATOS_CUDA(cudaMalloc(&p.row_ptr, (size_t)(nl + 1) * 4));
   ATOS_CUDA(cudaMalloc(&p.col, (size_t)std::max<int64_t>(ml, 1) * 4));
   if (where == ATOS_MEM_HOST) {
-    std::vector<uint32_t> rp((size_t)nl + 1);
-    for (int64_t i = 0; i <= nl; ++i) rp[(size_t)i] = (uint32_t)(row_ptr[v_begin + i] - e_begin);
-    ATOS_CUDA(cudaMemcpy(p.row_ptr, rp.data(), rp.size() * 4, cudaMemcpyHostToDevice));
+    // upload the int64 offsets as they are and narrow on the device (a host loop over n
+    // would cost more than the copy); col goes straight into its final buffer
+    int64_t* tmp = nullptr;
+    ATOS_CUDA(cudaMalloc(&tmp, (size_t)(nl + 1) * 8));
+    ATOS_CUDA(cudaMemcpy(tmp, row_ptr + v_begin, (size_t)(nl + 1) * 8, cudaMemcpyHostToDevice));
+    k_rebase_row_ptr<<<1024, 256>>>(tmp, p.row_ptr, nl + 1, e_begin);
+    g_launches++;
     if (ml) ATOS_CUDA(cudaMemcpy(p.col, col + e_begin, (size_t)ml * 4, cudaMemcpyHostToDevice));
+    ATOS_CUDA(cudaDeviceSynchronize());
+    cudaFree(tmp);
     return ATOS_OK;
   }
   // device input: rebase + narrow on the device
@@ -337,6 +343,8 @@ int upload_part_local(Part& p, const int64_t* row_ptr, const int32_t* col, int w
   return ATOS_OK;
 }
 
+// host CSR: offsets checked on the host (O(n)); col ids are checked on the device
+// after the upload (validate_uploaded_cols), which is far cheaper than a host pass over m
 static int validate_host_csr(int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col) {
   if (row_ptr[0] != 0 || row_ptr[n] != m) {
     set_error("row_ptr[0] must be 0 and row_ptr[n] must equal m");
@@ -347,11 +355,26 @@ static int validate_host_csr(int64_t n, int64_t m, const int64_t* row_ptr, const
       set_error("row_ptr is not non-decreasing at %lld", (long long)v);
       return ATOS_ERR_INVALID_ARG;
     }
-  for (int64_t e = 0; e < m; ++e)
-    if (col[e] < 0 || (int64_t)col[e] >= n) {
-      set_error("col[%lld] = %d out of range [0, %lld)", (long long)e, col[e], (long long)n);
-      return ATOS_ERR_INVALID_ARG;
+  (void)col;
+  return ATOS_OK;
+}
+
+static int validate_uploaded_cols(atos_csr* g) {
+  unsigned* bad = nullptr;
+  ATOS_CUDA(cudaMalloc(&bad, 4));
+  ATOS_CUDA(cudaMemset(bad, 0, 4));
+  for (auto& p : g->parts)
+    if (p.m_local) {
+      k_check_col<<<1024, 256>>>((const int32_t*)p.col, nullptr, p.m_local, g->n, bad);
+      g_launches++;
     }
+  unsigned h = 0;
+  ATOS_CUDA(cudaMemcpy(&h, bad, 4, cudaMemcpyDeviceToHost));
+  cudaFree(bad);
+  if (h) {
+    set_error("col has ids outside [0, n)");
+    return ATOS_ERR_INVALID_ARG;
+  }
   return ATOS_OK;
 }
 
@@ -484,6 +507,7 @@ int atos_csr_create(atos_csr** out, int64_t n, int64_t m, const int64_t* row_ptr
   g->m = m;
   g->num_parts = num_parts;
   int rc = num_parts == 1 ? create_single(g, row_ptr, col, where) : create_loopback_parts(g, row_ptr, col, where);
+  if (rc == ATOS_OK && where == ATOS_MEM_HOST) rc = validate_uploaded_cols(g);
   if (rc != ATOS_OK) {
     atos_csr_destroy(g);
     return rc;
