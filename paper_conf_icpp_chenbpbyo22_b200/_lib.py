@@ -10,7 +10,8 @@ import os
 import threading
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libatos.so")
+# ATOS_LIB selects an experimental variant build (tools only); the default is the in-tree library
+LIB_PATH = os.environ.get("ATOS_LIB") or os.path.join(HERE, "libatos.so")
 
 ATOS_OK = 0
 ERRORS = {
@@ -66,7 +67,7 @@ def load(build_if_missing: bool = True):
     with _lock:
         if _lib is not None:
             return _lib
-        if build_if_missing and os.path.exists("/usr/local/cuda/bin/nvcc"):
+        if build_if_missing and not os.environ.get("ATOS_LIB") and os.path.exists("/usr/local/cuda/bin/nvcc"):
             from . import build_lib
             build_lib.build()
         if not os.path.exists(LIB_PATH):

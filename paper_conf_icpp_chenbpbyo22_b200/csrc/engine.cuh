@@ -33,7 +33,13 @@
 namespace atos {
 
 enum { MODE_CTA = 0, MODE_WARP = 1, MODE_THREAD = 2 };
-constexpr int kU = 4;  // edges in flight per thread per expand iteration
+#ifndef ATOS_KU
+#define ATOS_KU 4
+#endif
+constexpr int kU = ATOS_KU;  // edges in flight per thread per expand iteration
+#ifndef ATOS_MINB
+#define ATOS_MINB 1
+#endif
 
 // ------------------------------------------------------------ big-task assist
 // A popped vertex whose degree exceeds big_threshold is not expanded by the
@@ -54,6 +60,18 @@ struct __align__(64) BigTask {
   uint32_t pad[9];
 };
 constexpr uint32_t kBigNextBits = 20, kBigChunkBits = 20;
+
+// Debug edge counters (build with -DATOS_DEBUG_COUNTS; runtime-enabled by ATOS_DEBUG_EDGES).
+#ifdef ATOS_DEBUG_COUNTS
+#define ATOS_DBG_EDGE(P, e) \
+  do {                      \
+    if ((P).dbg_edge) atomicAdd((P).dbg_edge + (e), 1u); \
+  } while (0)
+#else
+#define ATOS_DBG_EDGE(P, e) \
+  do {                      \
+  } while (0)
+#endif
 __host__ __device__ constexpr unsigned long long big_pack(uint32_t gen, uint32_t nchunks, uint32_t next) {
   return ((unsigned long long)(gen & 0xFFFFFFu) << 40) | ((unsigned long long)nchunks << 20) | next;
 }
@@ -430,7 +448,10 @@ __device__ __forceinline__ void flush_stats(const Ring& q, unsigned long long po
 
 // ------------------------------------------------------------------- kernel
 template <class App, int MODE, bool PERSIST>
-__global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) {
+#ifndef ATOS_MAXT
+#define ATOS_MAXT 1024
+#endif
+__global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_worker(App app, EngineParams P) {
   using Payload = typename App::Payload;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const uint32_t nwarps = blockDim.x >> 5;
@@ -472,25 +493,25 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
         const Payload p = payload_from<Payload>(((unsigned long long)s.ctr[46] << 32) | s.ctr[45]);
         my_edges += (r == 0) ? len : 0;
         for (uint32_t base = 0; base < len; base += G * kU) {
-          const uint32_t j0 = base + r * kU;  // kU consecutive edges per lane
+          // strided lanes (k * G + r): coalesced loads
           uint32_t w[kU];
           typename App::Token tk[kU];
 #pragma unroll
           for (int k = 0; k < kU; ++k)
-            if (j0 + k < len) {
-              w[k] = app.neighbor(st0 + j0 + k);
-              if (P.dbg_edge) atomicAdd(P.dbg_edge + st0 + j0 + k, 1u);
+            if (base + k * G + r < len) {
+              w[k] = app.neighbor(st0 + base + k * G + r);
+              ATOS_DBG_EDGE(P, st0 + base + k * G + r);
             }
 #pragma unroll
           for (int k = 0; k < kU; ++k)
-            if (j0 + k < len) tk[k] = app.pre(p, w[k]);
+            if (base + k * G + r < len) tk[k] = app.pre(p, w[k]);
           bool want[kU];
           uint32_t out[kU];
 #pragma unroll
           for (int k = 0; k < kU; ++k) {
             want[k] = false;
             out[k] = 0;
-            if (j0 + k < len) want[k] = app.post(p, w[k], tk[k], out[k]);
+            if (base + k * G + r < len) want[k] = app.post(p, w[k], tk[k], out[k]);
           }
           pusher.push_n<kU>(q, want, out, P.watchdog_ns);
         }
@@ -556,6 +577,34 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
           ob = l;
         }
         const uint32_t olo = __shfl_sync(0xffffffffu, ob, 0), ohi = __shfl_sync(0xffffffffu, ob, 1);
+        uint32_t w[kU];
+        typename App::Token tk[kU];
+        bool want[kU];
+        uint32_t out[kU];
+        if (olo == ohi) {
+          // fast path (warp-uniform): the warp's span lies in ONE row -- no owner search,
+          // strided lanes so every load instruction is one coalesced 128-byte access
+          const uint32_t st0 = s.start[olo] + (wfirst - s.off[olo]);
+          const uint32_t len = wlast - wfirst + 1;
+          const Payload p = s.pay[olo];
+#pragma unroll
+          for (int k = 0; k < kU; ++k)
+            if (k * 32 + lane_id() < len) {
+              w[k] = app.neighbor(st0 + k * 32 + lane_id());
+              ATOS_DBG_EDGE(P, st0 + k * 32 + lane_id());
+            }
+#pragma unroll
+          for (int k = 0; k < kU; ++k)
+            if (k * 32 + lane_id() < len) tk[k] = app.pre(p, w[k]);
+#pragma unroll
+          for (int k = 0; k < kU; ++k) {
+            want[k] = false;
+            out[k] = 0;
+            if (k * 32 + lane_id() < len) want[k] = app.post(p, w[k], tk[k], out[k]);
+          }
+          pusher.push_n<kU>(q, want, out, P.watchdog_ns);
+          continue;
+        }
         const uint32_t e0 = wfirst + lane_id() * kU;
         uint32_t o = olo;
         {
@@ -566,9 +615,8 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
           }
           o = l;
         }
-        uint32_t w[kU], own[kU];
+        uint32_t own[kU];
         bool val[kU];
-        typename App::Token tk[kU];
 #pragma unroll
         for (int k = 0; k < kU; ++k) {
           const uint32_t e = e0 + k;
@@ -578,14 +626,12 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
             own[k] = o;
             const uint32_t ce = s.start[o] + (e - s.off[o]);
             w[k] = app.neighbor(ce);
-            if (P.dbg_edge) atomicAdd(P.dbg_edge + ce, 1u);
+            ATOS_DBG_EDGE(P, ce);
           }
         }
 #pragma unroll
         for (int k = 0; k < kU; ++k)
           if (val[k]) tk[k] = app.pre(s.pay[own[k]], w[k]);
-        bool want[kU];
-        uint32_t out[kU];
 #pragma unroll
         for (int k = 0; k < kU; ++k) {
           want[k] = false;
@@ -600,25 +646,25 @@ __global__ void __launch_bounds__(1024) k_relax_worker(App app, EngineParams P) 
         const Payload p = s.pay[k];
         my_edges += (r == 0) ? dg : 0;
         for (uint32_t j = 0; j < dg; j += 32 * kU) {
-          const uint32_t j0 = j + r * kU;  // kU consecutive edges per lane
+          // strided lanes: each load instruction is one coalesced access
           uint32_t w[kU];
           typename App::Token tk[kU];
 #pragma unroll
           for (int k = 0; k < kU; ++k)
-            if (j0 + k < dg) {
-              w[k] = app.neighbor(st + j0 + k);
-              if (P.dbg_edge) atomicAdd(P.dbg_edge + st + j0 + k, 1u);
+            if (j + k * 32 + r < dg) {
+              w[k] = app.neighbor(st + j + k * 32 + r);
+              ATOS_DBG_EDGE(P, st + j + k * 32 + r);
             }
 #pragma unroll
           for (int k = 0; k < kU; ++k)
-            if (j0 + k < dg) tk[k] = app.pre(p, w[k]);
+            if (j + k * 32 + r < dg) tk[k] = app.pre(p, w[k]);
           bool want[kU];
           uint32_t out[kU];
 #pragma unroll
           for (int k = 0; k < kU; ++k) {
             want[k] = false;
             out[k] = 0;
-            if (j0 + k < dg) want[k] = app.post(p, w[k], tk[k], out[k]);
+            if (j + k * 32 + r < dg) want[k] = app.post(p, w[k], tk[k], out[k]);
           }
           pusher.push_n<kU>(q, want, out, P.watchdog_ns);
         }
