@@ -37,13 +37,16 @@ struct GhostView {
   void* ghost;
   uint32_t* touched;
   unsigned long long* ntouched;
-  __device__ __forceinline__ bool remote(uint32_t w) const { return ghost != nullptr && (w - vb) >= nl; }
+  __device__ __forceinline__ bool remote_dyn(uint32_t w) const { return ghost != nullptr && (w - vb) >= nl; }
   __device__ __forceinline__ void touch(uint32_t w) const {
     touched[atomicAdd(ntouched, 1ull)] = w;
   }
 };
 
-struct BfsApp {
+// PART (compile time): partitioned run (ghosts, local ids); false = single
+// partition, where every neighbour is local and vb == 0.
+template <bool PART>
+struct BfsAppT {
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
   const uint32_t* __restrict__ row_ptr;
@@ -54,6 +57,7 @@ struct BfsApp {
   unsigned long long pol_first, pol_last;
   GhostView gv;
 
+  __device__ __forceinline__ bool remote(uint32_t w) const { return PART && gv.remote_dyn(w); }
   __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
   __device__ __forceinline__ void prepare() {
     pol_first = policy_evict_first();
@@ -79,8 +83,8 @@ struct BfsApp {
   }
 
   __device__ __forceinline__ Token pre(const Payload nd, uint32_t w) const {
-    if (gv.remote(w)) return 0u;
-    return pre_local(w - gv.vb);
+    if (remote(w)) return 0u;
+    return pre_local(PART ? w - gv.vb : w);
   }
 
   // relax local vertex lw with candidate depth nd; true -> enqueue lw
@@ -117,14 +121,14 @@ struct BfsApp {
   }
 
   __device__ __forceinline__ bool post(const Payload nd, uint32_t w, Token tok, uint32_t& out) const {
-    if (gv.remote(w)) {
+    if (remote(w)) {
       // remote relaxation: min-combine into the ghost, list it on first touch this round
       uint32_t* g = (uint32_t*)gv.ghost + w;
       if (ld_relaxed(g) <= nd) return false;
       if (atomicMin(g, nd) == 0xFFFFFFFFu) gv.touch(w);
       return false;
     }
-    return relax_local(nd, w - gv.vb, tok, out);
+    return relax_local(nd, PART ? w - gv.vb : w, tok, out);
   }
 
   __device__ __forceinline__ bool relax(const Payload nd, uint32_t w, uint32_t& out) const {
@@ -143,7 +147,8 @@ struct BfsApp {
 // Activation (DESIGN.md R-PR-6): w is pushed iff its residue crosses eps from
 // below (old <= eps < old + delta, evaluated in the same fp64 rounding as the
 // atomic), which keeps "residue[v] > eps  =>  v queued or in flight".
-struct PrApp {
+template <bool PART>
+struct PrAppT {
   using Payload = double;  // delta = alpha * rho / deg(v)
   using Token = double;    // residue before our atomicAdd
   const uint32_t* __restrict__ row_ptr;
@@ -156,6 +161,7 @@ struct PrApp {
   uint32_t* dbg_expand;  // debug: per-vertex count of expanding pops
   GhostView gv;
 
+  __device__ __forceinline__ bool remote(uint32_t w) const { return PART && gv.remote_dyn(w); }
   __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
   __device__ __forceinline__ void prepare() { pol_first = policy_evict_first(); }
 
@@ -172,8 +178,8 @@ struct PrApp {
   }
 
   __device__ __forceinline__ Token pre(const Payload delta, uint32_t w) const {
-    if (gv.remote(w)) return 0.0;
-    return atomicAdd(res + (w - gv.vb), delta);
+    if (remote(w)) return 0.0;
+    return atomicAdd(res + (PART ? w - gv.vb : w), delta);
   }
   __device__ __forceinline__ bool crossing(const Payload delta, uint32_t lw, Token old, uint32_t& out) const {
     if (activate && old <= eps && old + delta > eps) {
@@ -183,12 +189,12 @@ struct PrApp {
     return false;
   }
   __device__ __forceinline__ bool post(const Payload delta, uint32_t w, Token old, uint32_t& out) const {
-    if (gv.remote(w)) {
+    if (remote(w)) {
       // remote mass: sum into the ghost, list it on first touch this round (delta > 0)
       if (atomicAdd((double*)gv.ghost + w, delta) == 0.0) gv.touch(w);
       return false;
     }
-    return crossing(delta, w - gv.vb, old, out);
+    return crossing(delta, PART ? w - gv.vb : w, old, out);
   }
   __device__ __forceinline__ bool relax(const Payload delta, uint32_t w, uint32_t& out) const {
     return post(delta, w, pre(delta, w), out);
@@ -197,5 +203,10 @@ struct PrApp {
     return crossing(delta, lw, atomicAdd(res + lw, delta), out);
   }
 };
+
+using BfsApp = BfsAppT<false>;
+using BfsPartApp = BfsAppT<true>;
+using PrApp = PrAppT<false>;
+using PrPartApp = PrAppT<true>;
 
 }  // namespace atos

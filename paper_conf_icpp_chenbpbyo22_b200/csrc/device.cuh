@@ -281,6 +281,7 @@ struct WarpPusher {
     uint32_t c = 0;
 #pragma unroll
     for (int k = 0; k < N; ++k) c += want[k] ? 1u : 0u;
+    if (!__any_sync(0xffffffffu, c != 0)) return;  // common case late in a run: nothing to push
     uint32_t incl = c;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {

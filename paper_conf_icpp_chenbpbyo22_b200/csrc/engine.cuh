@@ -37,6 +37,7 @@ enum { MODE_CTA = 0, MODE_WARP = 1, MODE_THREAD = 2 };
 #define ATOS_KU 4
 #endif
 constexpr int kU = ATOS_KU;  // edges in flight per thread per expand iteration
+constexpr uint32_t kCown = 2048;  // CTA mode: per-batch owner table of 32*kU-edge chunks
 #ifndef ATOS_MINB
 #define ATOS_MINB 1
 #endif
@@ -462,6 +463,8 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
   const GroupSmem<Payload>& s = wk.s;
   const uint32_t r = wk.r, G = wk.G;
   WarpPusher pusher = make_pusher(pushbuf);
+  // CTA mode: owner table after the group arena
+  uint32_t* cown = (uint32_t*)(smem_raw + (size_t)nwarps * kPushBuf * 4 + group_smem_bytes<Payload>(wk.K));
   unsigned long long my_pops = 0, my_edges = 0;
   const Ring& q = P.q;
   app.prepare();
@@ -562,12 +565,31 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
       // walks forward over its kU edges.  All col loads, then all prefilter
       // loads, then the decisions/atomics: kU memory chains in flight per lane.
       const uint32_t wspan = 32u * kU;
+      // owner of every wspan-edge chunk start, once per batch (a warp's span is
+      // one chunk, so its owner range comes from two table reads)
+      const uint32_t nchunk = (total + wspan - 1) / wspan;
+      const bool table = nchunk <= kCown;
+      if (table) {
+        for (uint32_t c = r; c < nchunk; c += G) {
+          const uint32_t e = c * wspan;
+          uint32_t l = 0, h = nready;
+          while (h - l > 1) {
+            const uint32_t mid = (l + h) >> 1;
+            if (s.off[mid] <= e) l = mid; else h = mid;
+          }
+          cown[c] = l;
+        }
+        __syncthreads();
+      }
       for (uint32_t base = 0; base < total; base += G * kU) {
         const uint32_t wfirst = base + (r & ~31u) * kU;
         if (wfirst >= total) continue;  // warp-uniform; no collective below is skipped by part of a warp
         const uint32_t wlast = min(wfirst + wspan, total) - 1;
         uint32_t ob = 0;
-        if (lane_id() < 2) {
+        if (table) {
+          const uint32_t c = wfirst / wspan;
+          ob = lane_id() == 0 ? cown[c] : (c + 1 < nchunk ? cown[c + 1] : nready - 1);
+        } else if (lane_id() < 2) {
           const uint32_t e = lane_id() == 0 ? wfirst : wlast;
           uint32_t l = 0, h = nready;
           while (h - l > 1) {
@@ -705,7 +727,7 @@ inline size_t relax_worker_smem(int mode, uint32_t block, uint32_t fetch) {
   uint32_t nwarps = block / 32;
   uint32_t K = mode == MODE_THREAD ? 32u * fetch : fetch;
   uint32_t groups = mode == MODE_CTA ? 1u : nwarps;
-  return (size_t)nwarps * kPushBuf * 4 + group_smem_bytes<Payload>(K) * groups;
+  return (size_t)nwarps * kPushBuf * 4 + group_smem_bytes<Payload>(K) * groups + (mode == MODE_CTA ? kCown * 4 : 0);
 }
 
 }  // namespace atos

@@ -492,7 +492,7 @@ __global__ void k_pr_init_edges_part(const uint32_t* __restrict__ row_ptr, const
       const uint32_t deg = __ldg(row_ptr + v + 1) - __ldg(row_ptr + v);
       const uint32_t w = __ldg(col + e);
       const double add = c / (double)deg;
-      if (gv.remote(w)) {
+      if (gv.remote_dyn(w)) {
         if (atomicAdd((double*)gv.ghost + w, add) == 0.0) gv.touch(w);
       } else {
         red_add_f64(res + (w - gv.vb), add);
@@ -619,7 +619,7 @@ int bfs_partitioned(atos_csr* g, int64_t src, uint32_t* depth_out, const Resolve
   cudaStream_t s = r.stream;
   const uint32_t P = g->comm ? (uint32_t)g->nranks : (uint32_t)g->num_parts;
   std::vector<PartRun> runs(g->parts.size());
-  std::vector<BfsApp> apps(g->parts.size());
+  std::vector<BfsPartApp> apps(g->parts.size());
   for (size_t i = 0; i < g->parts.size(); ++i) {
     Part& p = g->parts[i];
     const int64_t n = p.n_local;
@@ -645,10 +645,10 @@ int bfs_partitioned(atos_csr* g, int64_t src, uint32_t* depth_out, const Resolve
                                      has ? (uint32_t)(src - p.v_begin) : 0u, has ? 1 : 0, r.watchdog_ns);
     ++g_launches;
     p.ring_clean = false;
-    apps[i] = BfsApp{p.row_ptr, p.col, depth, r.dedupe, p.shadow.as<uint8_t>(), 0ull, 0ull, pr.gv};
+    apps[i] = BfsPartApp{p.row_ptr, p.col, depth, r.dedupe, p.shadow.as<uint8_t>(), 0ull, 0ull, pr.gv};
   }
   ATOS_CUDA(cudaGetLastError());
-  return run_rounds<BfsApp, uint32_t>(g, runs, apps, r, 0xFFFFFFFFu, st);
+  return run_rounds<BfsPartApp, uint32_t>(g, runs, apps, r, 0xFFFFFFFFu, st);
 }
 
 int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_out, const Resolved& r,
@@ -660,7 +660,7 @@ int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_out
     return ATOS_ERR_UNSUPPORTED;
   }
   std::vector<PartRun> runs(g->parts.size());
-  std::vector<PrApp> apps(g->parts.size());
+  std::vector<PrPartApp> apps(g->parts.size());
   const int gs = 148 * 8;
   for (size_t i = 0; i < g->parts.size(); ++i) {
     Part& p = g->parts[i];
@@ -696,10 +696,10 @@ int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_out
     }
     g_launches += 1;
     p.ring_clean = false;
-    apps[i] = PrApp{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, 1, nullptr, pr.gv};
+    apps[i] = PrPartApp{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, 1, nullptr, pr.gv};
   }
   ATOS_CUDA(cudaGetLastError());
-  ATOS_TRY((run_rounds<PrApp, double>(g, runs, apps, r, 0.0, st)));
+  ATOS_TRY((run_rounds<PrPartApp, double>(g, runs, apps, r, 0.0, st)));
   // finalize: rank / n_global, residual sum over all partitions (conservation)
   double total = 0.0;
   for (size_t i = 0; i < g->parts.size(); ++i) {
