@@ -359,14 +359,30 @@ struct Worker {
             else { *(unsigned long long*)&s.ctr[6] = b; s.ctr[4] = (uint32_t)(e - b); }
           }
         } else if (s.ctr[1] == 0) {
-          // bounded over-claim: at most the items visible at the tail
-          const unsigned long long h = ld_relaxed(&q.ctl->head.v);
+          // Claim.  Plenty of published work (>= 2K visible): one atomicAdd of K
+          // (a concurrent over-claim past the tail is filled by the ongoing pushes).
+          // Sparse queue: an exact CAS claim of what is visible, so no index past
+          // the tail is ever parked in a sleeping worker's pending list (that made
+          // late improvement cascades crawl one backoff period per item).
+          unsigned long long h = ld_relaxed(&q.ctl->head.v);
           const unsigned long long t = ld_relaxed(&q.ctl->tail.v);
           if (h < t) {
-            const unsigned long long amt = t - h < K ? t - h : K;
-            const unsigned long long b = atomicAdd(&q.ctl->head.v, amt);
-            *(unsigned long long*)&s.ctr[6] = b;
-            s.ctr[4] = (uint32_t)amt;
+            if (t - h >= 2ull * K) {
+              const unsigned long long b = atomicAdd(&q.ctl->head.v, (unsigned long long)K);
+              *(unsigned long long*)&s.ctr[6] = b;
+              s.ctr[4] = K;
+            } else {
+              for (int tries = 0; tries < 4 && h < t; ++tries) {
+                const unsigned long long amt = t - h < K ? t - h : K;
+                const unsigned long long old = atomicCAS(&q.ctl->head.v, h, h + amt);
+                if (old == h) {
+                  *(unsigned long long*)&s.ctr[6] = h;
+                  s.ctr[4] = (uint32_t)amt;
+                  break;
+                }
+                h = old;
+              }
+            }
           }
         }
       }
@@ -412,7 +428,7 @@ struct Worker {
           }
           tl_sample(P);
           __nanosleep(backoff);
-          backoff = backoff < 2048 ? backoff * 2 : 2048;
+          backoff = backoff < 1024 ? backoff * 2 : 1024;
         }
       }
       group_sync<MODE>();

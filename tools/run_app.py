@@ -42,7 +42,8 @@ def main():
         if tlb is not None:
             t = atos.timeline_table(tlb, st)
             n = t.shape[0]
-            idx = sorted(set([int(i * (n - 1) / 24) for i in range(25)])) if n else []
+            nrow = int(os.environ.get("TL_ROWS", "25"))
+            idx = sorted(set([int(i * (n - 1) / (nrow - 1)) for i in range(nrow)])) if n else []
             print("  t_us      done        tail        head")
             for i in idx:
                 print(f"  {t[i,0].item()/1e3:8.1f} {t[i,1].item():11d} {t[i,2].item():11d} {t[i,3].item():11d}")
