@@ -92,8 +92,9 @@ typedef struct {
 typedef struct {
     uint32_t struct_size;       /* = sizeof(atos_cfg); set by atos_cfg_default */
     int      persistent;        /* 1 persistent kernel (default), 0 discrete per-frontier launches */
-    int      worker;            /* 1 thread, 32 warp, 64..1024 CTA; 0 = per-app default */
-    int      fetch_size;        /* items per pop per worker (FETCH_SIZE); 0 = default */
+    int      worker;            /* 1 thread, 32 warp, 64..1024 CTA; 0 = per-app default (CTA 256; colouring 512) */
+    int      fetch_size;        /* items per pop per worker (FETCH_SIZE); 0 = default (CTA: worker size,
+                                   colouring min(worker,128); warp 8; thread 1) */
     int      num_blocks;        /* 0 = occupancy max (persistent) / proportional to the frontier (discrete) */
     int      block_threads;     /* threads per block for thread/warp workers; 0 = 256 */
     int      dedupe;            /* 1 (default): in-queue bitmap, a vertex is queued at most once at a time;

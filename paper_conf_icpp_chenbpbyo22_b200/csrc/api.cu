@@ -57,13 +57,16 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
   }
   r->persistent = d.persistent ? 1 : 0;
   r->worker = d.worker;
-  if (r->worker == 0) r->worker = (app == 'c') ? 32 : 256;
+  // defaults measured on B200: CTA workers with load-balancing search
+  // win for all three apps, including colouring (512 threads, fetch 128)
+  if (r->worker == 0) r->worker = (app == 'c') ? 512 : 256;
   if (!(r->worker == 1 || r->worker == 32 || (r->worker >= 64 && r->worker <= 1024 && r->worker % 32 == 0))) {
     set_error("worker must be 1, 32 or a multiple of 32 in [64, 1024] (got %d)", r->worker);
     return ATOS_ERR_INVALID_ARG;
   }
   r->fetch = d.fetch_size;
-  if (r->fetch == 0) r->fetch = (r->worker >= 64) ? r->worker : (r->worker == 32 ? 8 : 1);
+  if (r->fetch == 0)
+    r->fetch = (r->worker >= 64) ? (app == 'c' ? std::min(r->worker, 128) : r->worker) : (r->worker == 32 ? 8 : 1);
   if (r->fetch < 1 || r->fetch > 4096) {
     set_error("fetch_size must be in [1, 4096] (got %d)", r->fetch);
     return ATOS_ERR_INVALID_ARG;
