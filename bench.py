@@ -374,6 +374,29 @@ def run_apps(args, dev, peak):
                     "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak}
     del csr, g, out
     torch.cuda.empty_cache()
+    # ---- C2: high-diameter mesh, persistent vs discrete kernel strategy
+    from paper_conf_icpp_chenbpbyo22_b200 import gen
+    R = C = args.mesh_side
+    g = gen.mesh(R, C, device=dev)
+    csr = atos.CSR.from_graph(g)
+    src = gen.mesh_centre_source(g, R, C)
+    out = torch.empty(g.n, dtype=torch.int32, device=dev)
+    mres = {"config": f"C2: {R}x{C} 4-neighbour mesh (n={g.n}, m={g.m}), centre source"}
+    for name, knobs in (("persistent", dict()), ("discrete", dict(persistent=0))):
+        atos.bfs(csr, src, out=out, **knobs)
+        ms = []
+        for _ in range(args.app_steps):
+            flush_l2(flush)
+            torch.cuda.synchronize()
+            _, st = atos.bfs(csr, src, out=out, **knobs)
+            ms.append(st["kernel_ms"])
+        levels = int(out.max().item()) + 1
+        mres[name] = {"ms": float(np.mean(ms)), "levels": levels, "us_per_level": 1e3 * float(np.mean(ms)) / levels,
+                      "gteps": g.m / (float(np.mean(ms)) / 1e3) / 1e9, "launches": int(st["rounds"])}
+    mres["persistent_speedup"] = mres["discrete"]["ms"] / mres["persistent"]["ms"]
+    res["mesh_c2"] = mres
+    del csr, g, out
+    torch.cuda.empty_cache()
     return res
 
 
@@ -387,6 +410,7 @@ def main():
     ap.add_argument("--pr-scale", type=int, default=22)
     ap.add_argument("--gc-scale", type=int, default=20)
     ap.add_argument("--app-steps", type=int, default=3)
+    ap.add_argument("--mesh-side", type=int, default=4900)
     ap.add_argument("--worker", type=int, default=256)
     ap.add_argument("--fetch", type=int, default=256)
     ap.add_argument("--no-apps", action="store_true")
