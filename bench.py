@@ -274,6 +274,8 @@ def run_atos(args, ws, rank, local):
                    "mean_reached_vertices": float(np.mean(verts)), "mean_reached_edges": float(np.mean(edges))},
         "roofline": roofline, "clocks": clocks, "gpu_launches": int(launches),
     }
+    if ws == 1 and not args.no_bsp:
+        line["bsp"] = {"bfs_c5": bsp_bfs(csr, sources, src_info, out, flush, ms_per_step)}
     if rank == 0 and ws == 1:
         line["e2e"] = e2e_bfs(args, g, sources, src_info, knobs, local)
         if not args.no_cpu:
@@ -284,6 +286,24 @@ def run_atos(args, ws, rank, local):
         line["e2e"] = None
     if rank == 0:
         print(json.dumps(line), flush=True)
+
+
+def bsp_bfs(csr, sources, src_info, out, flush, atos_ms):
+    """The bulk-synchronous baseline (Alg.1, atos_bfs_bsp) on the same graph and sources, same
+    L2-flush protocol: the paper's Atos-vs-BSP comparison (Table 1) on this B200."""
+    import paper_conf_icpp_chenbpbyo22_b200 as atos
+    atos.bfs_bsp(csr, sources[0], out=out)
+    ms, edges, rounds = [], [], []
+    for k in range(len(sources)):
+        flush_l2(flush)
+        torch.cuda.synchronize()
+        _, st = atos.bfs_bsp(csr, sources[k], out=out)
+        ms.append(st["kernel_ms"])
+        rounds.append(st["rounds"])
+        edges.append(src_info[k][1])
+    m = float(np.mean(ms))
+    return {"ms": m, "gteps": float(np.sum(edges) / (np.sum(ms) / 1e3) / 1e9), "levels_mean": float(np.mean(rounds)),
+            "atos_speedup": m / atos_ms, "note": "Alg.1 level-synchronous, edge-balanced advance + host barrier per level"}
 
 
 def e2e_bfs(args, g, sources, src_info, knobs, local, steps=2):
@@ -320,6 +340,23 @@ def cpu_baseline(g, sources, src_info):
             "seconds": dt}
 
 
+def bsp_app(call, flush, g, atos_ms, steps=2):
+    """Time a BSP baseline call (stats.kernel_ms, L2 flushed before each step) next to the Atos number."""
+    call()
+    ms, st = [], None
+    for _ in range(steps):
+        flush_l2(flush)
+        torch.cuda.synchronize()
+        _, st = call()
+        ms.append(st["kernel_ms"])
+    m = float(np.mean(ms))
+    out = {"ms": m, "rounds": int(st["rounds"]), "pops_per_n": st["pops"] / g.n, "edges_per_m": st["edges"] / g.m,
+           "atos_speedup": m / atos_ms}
+    if st.get("colors_used"):
+        out["colors"] = int(st["colors_used"])
+    return out
+
+
 def run_apps(args, dev, peak):
     """PageRank (C3) and colouring (C4) ms to converge, each with its roofline numbers."""
     import paper_conf_icpp_chenbpbyo22_b200 as atos
@@ -347,6 +384,9 @@ def run_apps(args, dev, peak):
                        "pops_per_n": float(np.mean(pops)) / g.n, "edge_relaxations_per_m": float(np.mean(edges)) / g.m,
                        "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
                        "traffic": profile_traffic("pr_worker")}
+    if not args.no_bsp:
+        res["pagerank"]["bsp"] = bsp_app(lambda: atos.pagerank_bsp(csr, 0.85, 1e-6, out=out), flush, g,
+                                         float(np.mean(ms)))
     del csr, g, out
     torch.cuda.empty_cache()
     # ---- colouring on C4
@@ -368,10 +408,12 @@ def run_apps(args, dev, peak):
     wm = float(np.mean(wms))
     alg = GC_BYTES_PER_TASK * np.mean(pops) + GC_BYTES_PER_EDGE * np.mean(edges)
     res["color"] = {"config": f"C4: Kronecker scale {args.gc_scale} ef 64 seed 4 (n={g.n}, m={g.m}), seed 1, "
-                              "CTA worker 512 / fetch 128 (library default)",
+                              "CTA worker 1024 / fetch 128 (library default)",
                     "ms_to_converge": float(np.mean(ms)), "ms_min": float(np.min(ms)), "worker_ms": wm,
                     "colors": int(np.max(cols)), "tasks_per_n": float(np.mean(pops)) / g.n,
                     "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak}
+    if not args.no_bsp:
+        res["color"]["bsp"] = bsp_app(lambda: atos.color_bsp(csr, 1, out=out), flush, g, float(np.mean(ms)))
     del csr, g, out
     torch.cuda.empty_cache()
     # ---- C2: high-diameter mesh, persistent vs discrete kernel strategy
@@ -394,6 +436,9 @@ def run_apps(args, dev, peak):
         mres[name] = {"ms": float(np.mean(ms)), "levels": levels, "us_per_level": 1e3 * float(np.mean(ms)) / levels,
                       "gteps": g.m / (float(np.mean(ms)) / 1e3) / 1e9, "launches": int(st["rounds"])}
     mres["persistent_speedup"] = mres["discrete"]["ms"] / mres["persistent"]["ms"]
+    if not args.no_bsp:
+        mres["bsp"] = bsp_app(lambda: atos.bfs_bsp(csr, src, out=out), flush, g, mres["persistent"]["ms"])
+        mres["bsp"]["us_per_level"] = 1e3 * mres["bsp"]["ms"] / mres["bsp"]["rounds"]
     res["mesh_c2"] = mres
     del csr, g, out
     torch.cuda.empty_cache()
@@ -415,6 +460,7 @@ def main():
     ap.add_argument("--fetch", type=int, default=256)
     ap.add_argument("--no-apps", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-bsp", action="store_true", help="skip the bulk-synchronous baselines (atos_*_bsp)")
     args = ap.parse_args()
     if args.warmup < 3:
         log("[bench] warmup raised to 3 (timing rules)")

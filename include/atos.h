@@ -92,7 +92,8 @@ typedef struct {
 typedef struct {
     uint32_t struct_size;       /* = sizeof(atos_cfg); set by atos_cfg_default */
     int      persistent;        /* 1 persistent kernel (default), 0 discrete per-frontier launches */
-    int      worker;            /* 1 thread, 32 warp, 64..1024 CTA; 0 = per-app default (CTA 256; colouring 512) */
+    int      worker;            /* 1 thread, 32 warp, 64..1024 CTA; 0 = per-app default (CTA: BFS 256, PageRank 512,
+                                   colouring 1024) */
     int      fetch_size;        /* items per pop per worker (FETCH_SIZE); 0 = default (CTA: worker size,
                                    colouring min(worker,128); warp 8; thread 1) */
     int      num_blocks;        /* 0 = occupancy max (persistent) / proportional to the frontier (discrete) */
@@ -174,6 +175,35 @@ ATOS_API int atos_pagerank(const atos_csr* g, double alpha, double eps, double* 
  * single partition only (ATOS_ERR_UNSUPPORTED otherwise).
  */
 ATOS_API int atos_color(const atos_csr* g, uint64_t seed, int32_t* color_out, const atos_cfg* cfg);
+
+/* ---- bulk-synchronous baselines (the paper's comparison point) ----------- */
+/*
+ * The BSP versions of the three applications, run on the same handle and
+ * with the same result conventions, so Atos can be compared against BSP on
+ * the same device (the paper's Table 1 comparison):
+ *  - atos_bfs_bsp:      Alg.1, level-synchronous; depth_out exact
+ *                       (bit-identical to atos_bfs).
+ *  - atos_pagerank_bsp: Alg.3: per iteration every frontier
+ *                       vertex pushes its whole residue, then the frontier is
+ *                       rebuilt as {v : residue[v] > eps}; same init, output
+ *                       scale and error bound as atos_pagerank.
+ *  - atos_color_bsp:    Alg.5: assign kernel, barrier, conflict
+ *                       kernel; a conflict re-queues the lower-priority
+ *                       endpoint (priority splitmix64(seed ^ v)), or both
+ *                       endpoints with cfg->conflict_policy = 1 (the literal
+ *                       Alg.5, which may not terminate: set timeout_s).
+ * Used cfg fields: stream, stats, out_where, timeout_s, validate
+ * (colouring), conflict_policy (colouring); the scheduler knobs are ignored.
+ * stats: pops = frontier items processed (colouring: assign + check),
+ * rounds = iterations (barriers), edges = neighbour entries visited.
+ * Single partition only (ATOS_ERR_UNSUPPORTED otherwise).  Each iteration
+ * ends with a host round trip reading the next frontier's size (the paper's
+ * cudaDeviceSynchronize() barrier).
+ */
+ATOS_API int atos_bfs_bsp(const atos_csr* g, int64_t src, uint32_t* depth_out, const atos_cfg* cfg);
+ATOS_API int atos_pagerank_bsp(const atos_csr* g, double alpha, double eps, double* rank_out,
+                               const atos_cfg* cfg);
+ATOS_API int atos_color_bsp(const atos_csr* g, uint64_t seed, int32_t* color_out, const atos_cfg* cfg);
 
 /* ---- multi-process (one process per GPU, e.g. torchrun) ------------------ */
 

@@ -15,7 +15,7 @@ import torch
 from . import _lib
 from ._lib import UNREACHED, Stats, default_cfg
 
-__all__ = ["CSR", "bfs", "pagerank", "color", "UNREACHED", "launches", "partition_range", "Comm"]
+__all__ = ["CSR", "bfs", "pagerank", "color", "bfs_bsp", "pagerank_bsp", "color_bsp", "UNREACHED", "launches", "partition_range", "Comm"]
 
 
 def _ptr(t: torch.Tensor) -> ctypes.c_void_p:
@@ -119,6 +119,28 @@ def color(g: CSR, seed: int = 1, out: torch.Tensor | None = None, stream=None, *
     if out is None:
         out = torch.empty(g.n, dtype=torch.int32, device=f"cuda:{g.device}")
     return _run("atos_color", g, out, (ctypes.c_uint64(seed & (2**64 - 1)),), stream, knobs)
+
+
+def bfs_bsp(g: CSR, src: int, out: torch.Tensor | None = None, stream=None, **knobs):
+    """Bulk-synchronous BFS baseline (Alg.1).  Same result as bfs()."""
+    if out is None:
+        out = torch.empty(g.n, dtype=torch.int32, device=f"cuda:{g.device}")
+    return _run("atos_bfs_bsp", g, out, (int(src),), stream, knobs)
+
+
+def pagerank_bsp(g: CSR, alpha: float = 0.85, eps: float = 1e-6, out: torch.Tensor | None = None, stream=None,
+                 **knobs):
+    """Bulk-synchronous PageRank baseline (Alg.3).  Same output scale and bound as pagerank()."""
+    if out is None:
+        out = torch.empty(g.n, dtype=torch.float64, device=f"cuda:{g.device}")
+    return _run("atos_pagerank_bsp", g, out, (float(alpha), float(eps)), stream, knobs)
+
+
+def color_bsp(g: CSR, seed: int = 1, out: torch.Tensor | None = None, stream=None, **knobs):
+    """Bulk-synchronous speculative colouring baseline (Alg.5)."""
+    if out is None:
+        out = torch.empty(g.n, dtype=torch.int32, device=f"cuda:{g.device}")
+    return _run("atos_color_bsp", g, out, (ctypes.c_uint64(seed & (2**64 - 1)),), stream, knobs)
 
 
 def timeline_table(timeline: torch.Tensor, stats: dict):

@@ -28,7 +28,7 @@ EXPORTS = [
     "atos_cfg_default", "atos_csr_create", "atos_csr_destroy", "atos_csr_info", "atos_bfs",
     "atos_pagerank", "atos_color", "atos_comm_unique_id", "atos_comm_create", "atos_comm_destroy",
     "atos_csr_create_part", "atos_partition_range", "atos_last_error", "atos_version",
-    "atos_kernel_launches",
+    "atos_kernel_launches", "atos_bfs_bsp", "atos_pagerank_bsp", "atos_color_bsp",
 ]
 
 
@@ -83,6 +83,9 @@ def load(build_if_missing: bool = True):
             "atos_bfs": (i32, [P, i64, P, ctypes.POINTER(Cfg)]),
             "atos_pagerank": (i32, [P, dbl, dbl, P, ctypes.POINTER(Cfg)]),
             "atos_color": (i32, [P, u64, P, ctypes.POINTER(Cfg)]),
+            "atos_bfs_bsp": (i32, [P, i64, P, ctypes.POINTER(Cfg)]),
+            "atos_pagerank_bsp": (i32, [P, dbl, dbl, P, ctypes.POINTER(Cfg)]),
+            "atos_color_bsp": (i32, [P, u64, P, ctypes.POINTER(Cfg)]),
             "atos_comm_unique_id": (i32, [P, sz]),
             "atos_comm_create": (i32, [ctypes.POINTER(P), i32, i32, P, sz, i32]),
             "atos_comm_destroy": (None, [P]),

@@ -58,8 +58,9 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
   r->persistent = d.persistent ? 1 : 0;
   r->worker = d.worker;
   // defaults measured on B200: CTA workers with load-balancing search
-  // win for all three apps, including colouring (512 threads, fetch 128)
-  if (r->worker == 0) r->worker = (app == 'c') ? 512 : 256;
+  // win for all three apps (tools/sweep.py, gpurun_out sweep: BFS C5 256/256, PageRank C3 512/512,
+  // colouring C4 1024/128)
+  if (r->worker == 0) r->worker = (app == 'c') ? 1024 : (app == 'p' ? 512 : 256);
   if (!(r->worker == 1 || r->worker == 32 || (r->worker >= 64 && r->worker <= 1024 && r->worker % 32 == 0))) {
     set_error("worker must be 1, 32 or a multiple of 32 in [64, 1024] (got %d)", r->worker);
     return ATOS_ERR_INVALID_ARG;
@@ -197,10 +198,12 @@ int stream_wait(cudaStream_t s, double timeout_s) {
     return ATOS_OK;
   }
   auto t0 = std::chrono::steady_clock::now();
-  while (true) {
+  for (uint64_t polls = 0;; ++polls) {
     cudaError_t e = cudaStreamQuery(s);
     if (e == cudaSuccess) return ATOS_OK;
     if (e != cudaErrorNotReady) ATOS_CUDA(e);
+    // busy-poll first: a discrete per-frontier launch lasts microseconds and a sleep would dominate it
+    if (polls < 20000) continue;
     double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
     if (el > timeout_s * 1.5 + 1.0) {
       set_error("stream did not finish within timeout_s=%.3f", timeout_s);
@@ -414,7 +417,8 @@ void destroy_part(Part& p) {
   p.row_ptr = nullptr;
   p.col = nullptr;
   DevBuf* bufs[] = {&p.ring, &p.ctl, &p.big, &p.bitmap, &p.shadow, &p.vbuf_a, &p.vbuf_b, &p.vbuf_c, &p.scratch,
-                    &p.ghost_a, &p.ghost_b, &p.touched, &p.outbox, &p.inbox, &p.out_val, &p.in_val, &p.pack};
+                    &p.ghost_a, &p.ghost_b, &p.touched, &p.outbox, &p.inbox, &p.out_val, &p.in_val, &p.pack,
+                    &p.bsp_fa, &p.bsp_fb, &p.bsp_off, &p.bsp_tmp, &p.bsp_ctr};
   for (DevBuf* b : bufs) b->release();
   if (p.host_pinned) cudaFreeHost(p.host_pinned);
   p.host_pinned = nullptr;
@@ -629,6 +633,99 @@ int atos_color(const atos_csr* gc, uint64_t seed, int32_t* color_out, const atos
   if (g->n == 0) return ATOS_OK;
   int rc = run_with_output<int32_t>(g, color_out, g->n, r, g->parts[0].vbuf_c,
                                     [&](int32_t* d) { return color_single(g, g->parts[0], seed, d, r, st); });
+  const double ms = tm.stop();
+  if (rc == ATOS_OK && r.stats) {
+    local.kernel_ms = ms;
+    *r.stats = local;
+  }
+  return rc;
+}
+
+// ---- bulk-synchronous baselines (bsp.cu) ----------------
+int atos_bfs_bsp(const atos_csr* gc, int64_t src, uint32_t* depth_out, const atos_cfg* cfg) {
+  atos_csr* g = const_cast<atos_csr*>(gc);
+  if (!g || !depth_out) {
+    set_error("atos_bfs_bsp: null argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (src < 0 || src >= g->n) {
+    set_error("atos_bfs_bsp: src %lld out of range [0, %lld)", (long long)src, (long long)g->n);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (g->comm || g->num_parts > 1) {
+    set_error("atos_bfs_bsp: the BSP baseline runs on a single partition only");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  Resolved r;
+  ATOS_TRY(resolve_cfg(cfg, 'b', &r));
+  std::lock_guard<std::mutex> lk(g->mu);
+  DeviceGuard dg(g->device);
+  atos_stats local{};
+  atos_stats* st = r.stats ? &local : nullptr;
+  CallTimer tm(r.stream);
+  if (g->n == 0) return ATOS_OK;
+  int rc = run_with_output<uint32_t>(g, depth_out, g->n, r, g->parts[0].vbuf_c,
+                              [&](uint32_t* d) { return bfs_bsp_single(g, g->parts[0], src, d, r, st); });
+  const double ms = tm.stop();
+  if (rc == ATOS_OK && r.stats) {
+    local.kernel_ms = ms;
+    *r.stats = local;
+  }
+  return rc;
+}
+
+int atos_pagerank_bsp(const atos_csr* gc, double alpha, double eps, double* rank_out, const atos_cfg* cfg) {
+  atos_csr* g = const_cast<atos_csr*>(gc);
+  if (!g || !rank_out) {
+    set_error("atos_pagerank_bsp: null argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (!(alpha > 0.0 && alpha < 1.0) || !(eps > 0.0)) {
+    set_error("atos_pagerank_bsp: alpha must be in (0,1) and eps > 0 (alpha=%g eps=%g)", alpha, eps);
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (g->comm || g->num_parts > 1) {
+    set_error("atos_pagerank_bsp: the BSP baseline runs on a single partition only");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  Resolved r;
+  ATOS_TRY(resolve_cfg(cfg, 'p', &r));
+  std::lock_guard<std::mutex> lk(g->mu);
+  DeviceGuard dg(g->device);
+  atos_stats local{};
+  atos_stats* st = r.stats ? &local : nullptr;
+  CallTimer tm(r.stream);
+  if (g->n == 0) return ATOS_OK;
+  int rc = run_with_output<double>(g, rank_out, g->n, r, g->parts[0].vbuf_c,
+                              [&](double* d) { return pagerank_bsp_single(g, g->parts[0], alpha, eps, d, r, st); });
+  const double ms = tm.stop();
+  if (rc == ATOS_OK && r.stats) {
+    local.kernel_ms = ms;
+    *r.stats = local;
+  }
+  return rc;
+}
+
+int atos_color_bsp(const atos_csr* gc, uint64_t seed, int32_t* color_out, const atos_cfg* cfg) {
+  atos_csr* g = const_cast<atos_csr*>(gc);
+  if (!g || !color_out) {
+    set_error("atos_color_bsp: null argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (g->comm || g->num_parts > 1) {
+    set_error("atos_color_bsp: the BSP baseline runs on a single partition only");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  Resolved r;
+  ATOS_TRY(resolve_cfg(cfg, 'c', &r));
+  std::lock_guard<std::mutex> lk(g->mu);
+  DeviceGuard dg(g->device);
+  atos_stats local{};
+  atos_stats* st = r.stats ? &local : nullptr;
+  CallTimer tm(r.stream);
+  if (g->n == 0) return ATOS_OK;
+  int rc = run_with_output<int32_t>(g, color_out, g->n, r, g->parts[0].vbuf_c,
+                              [&](int32_t* d) { return color_bsp_single(g, g->parts[0], seed, d, r, st); });
   const double ms = tm.stop();
   if (rc == ATOS_OK && r.stats) {
     local.kernel_ms = ms;

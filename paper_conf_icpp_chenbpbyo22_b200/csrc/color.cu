@@ -491,24 +491,50 @@ static int launch_color_kernel(K kern_p, K kern_d, const ColorCtx& c, EnginePara
   return ATOS_OK;
 }
 
+// cfg.validate: reject a non-symmetric CSR (R-GC-8).  Shared with the BSP baseline (bsp.cu).
+int check_symmetric_if(Part& p, const Resolved& r) {
+  if (!r.validate) return ATOS_OK;
+  cudaStream_t s = r.stream;
+  unsigned* bad = nullptr;
+  ATOS_CUDA(cudaMalloc(&bad, 4));
+  ATOS_CUDA(cudaMemsetAsync(bad, 0, 4, s));
+  k_check_symmetric<<<1184, 256, 0, s>>>(p.row_ptr, p.col, (uint32_t)p.n_local, bad);
+  g_launches++;
+  unsigned hb = 0;
+  ATOS_CUDA(cudaMemcpyAsync(&hb, bad, 4, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  cudaFree(bad);
+  if (hb) {
+    set_error("atos_color: CSR is not symmetric");
+    return ATOS_ERR_NOT_SYMMETRIC;
+  }
+  return ATOS_OK;
+}
+
+// colours used (max + 1); fails if a vertex is left uncoloured.
+int color_count(Part& p, const int32_t* color, int64_t* used, cudaStream_t s) {
+  const uint32_t n = (uint32_t)p.n_local;
+  ATOS_TRY(p.scratch.ensure(64));
+  unsigned long long* mx = p.scratch.as<unsigned long long>();
+  unsigned* bad = (unsigned*)(mx + 1);
+  ATOS_CUDA(cudaMemsetAsync(mx, 0, 16, s));
+  k_color_max<<<592, 256, 0, s>>>(color, n, mx, bad);
+  g_launches++;
+  unsigned long long hm[2] = {0, 0};
+  ATOS_CUDA(cudaMemcpyAsync(hm, mx, 16, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  if ((unsigned)hm[1]) {
+    set_error("colouring left a vertex uncoloured");
+    return ATOS_ERR_CUDA;
+  }
+  *used = n ? (int64_t)hm[0] + 1 : 0;
+  return ATOS_OK;
+}
+
 int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Resolved& r, atos_stats* st) {
   cudaStream_t s = r.stream;
   const uint32_t n = (uint32_t)p.n_local;
-  if (r.validate) {
-    unsigned* bad = nullptr;
-    ATOS_CUDA(cudaMalloc(&bad, 4));
-    ATOS_CUDA(cudaMemsetAsync(bad, 0, 4, s));
-    k_check_symmetric<<<1184, 256, 0, s>>>(p.row_ptr, p.col, n, bad);
-    g_launches++;
-    unsigned hb = 0;
-    ATOS_CUDA(cudaMemcpyAsync(&hb, bad, 4, cudaMemcpyDeviceToHost, s));
-    ATOS_CUDA(cudaStreamSynchronize(s));
-    cudaFree(bad);
-    if (hb) {
-      set_error("atos_color: CSR is not symmetric");
-      return ATOS_ERR_NOT_SYMMETRIC;
-    }
-  }
+  ATOS_TRY(check_symmetric_if(p, r));
   // assign and check tasks of one vertex can both be queued: 2n outstanding + slack
   const uint64_t want = r.queue_capacity ? r.queue_capacity : std::max<uint64_t>(4ull * n, 4096);
   ATOS_TRY(ensure_queue(p, pow2_ceil(want), s));
@@ -569,19 +595,9 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   if (st) st->worker_ms += wt.elapsed();
   rc = finish_queue(p, s, st, "color");
   if (rc != ATOS_OK) return rc;
-  unsigned long long* mx = p.scratch.as<unsigned long long>();
-  unsigned* bad = (unsigned*)(mx + 1);
-  ATOS_CUDA(cudaMemsetAsync(mx, 0, 16, s));
-  k_color_max<<<592, 256, 0, s>>>(color, n, mx, bad);
-  g_launches++;
-  unsigned long long hm[2] = {0, 0};
-  ATOS_CUDA(cudaMemcpyAsync(hm, mx, 16, cudaMemcpyDeviceToHost, s));
-  ATOS_CUDA(cudaStreamSynchronize(s));
-  if ((unsigned)hm[1]) {
-    set_error("colouring left a vertex uncoloured");
-    return ATOS_ERR_CUDA;
-  }
-  if (st) st->colors_used = n ? (int64_t)hm[0] + 1 : 0;
+  int64_t used = 0;
+  ATOS_TRY(color_count(p, color, &used, s));
+  if (st) st->colors_used = used;
   return ATOS_OK;
 }
 

@@ -52,6 +52,7 @@ struct Part {
   // cached workspaces (grow-only, reused across calls)
   DevBuf ring, ctl, big, bitmap, shadow, vbuf_a, vbuf_b, vbuf_c, scratch;
   DevBuf ghost_a, ghost_b, touched, outbox, inbox, out_val, in_val, pack;
+  DevBuf bsp_fa, bsp_fb, bsp_off, bsp_tmp, bsp_ctr;  // BSP baselines (bsp.cu)
   uint64_t ring_cap = 0;
   void* host_pinned = nullptr;      // 4 KB pinned scratch for control-block reads
   bool ring_clean = false;          // every ring slot is EMPTY
@@ -187,6 +188,16 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
                     const Resolved& r, atos_stats* st);
 int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color_dev, const Resolved& r,
                  atos_stats* st);
+// bulk-synchronous baselines (bsp.cu): Alg.1 / Alg.3 / Alg.5
+int bfs_bsp_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth_dev, const Resolved& r, atos_stats* st);
+int pagerank_bsp_single(atos_csr* g, Part& p, double alpha, double eps, double* rank_dev, const Resolved& r,
+                        atos_stats* st);
+int color_bsp_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color_dev, const Resolved& r, atos_stats* st);
+// helpers shared by the asynchronous and BSP paths
+int pr_init_state(Part& p, double alpha, double* rank, double* res, cudaStream_t s);
+int pr_finalize(Part& p, double* rank, const double* res, double* h_sum, cudaStream_t s);
+int check_symmetric_if(Part& p, const Resolved& r);
+int color_count(Part& p, const int32_t* color, int64_t* used, cudaStream_t s);
 // partitioned solvers (dist.cu)
 int bfs_partitioned(atos_csr* g, int64_t src, uint32_t* depth_dev, const Resolved& r, atos_stats* st);
 int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_dev, const Resolved& r,

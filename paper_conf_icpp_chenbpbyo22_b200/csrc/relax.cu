@@ -299,6 +299,35 @@ int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolve
 }
 
 // ---------------------------------------------------------------- PageRank
+// Alg.3 init (R-PR-init): rank = 1 - alpha, residue[w] += (1-alpha)*alpha/deg(v)
+// over every edge v -> w.  Shared by the asynchronous path and the BSP baseline (bsp.cu).
+int pr_init_state(Part& p, double alpha, double* rank, double* res, cudaStream_t s) {
+  const int64_t n = p.n_local;
+  const int gs = 148 * 8;
+  k_pr_init_vertices<<<gs, 256, 0, s>>>(rank, res, n, 1.0 - alpha);
+  g_launches++;
+  if (p.m_local > 0) {
+    k_pr_init_edges<<<gs * 2, 256, 0, s>>>(p.row_ptr, p.col, res, (uint32_t)n, (uint32_t)p.m_local,
+                                            (1.0 - alpha) * alpha);
+    g_launches++;
+  }
+  ATOS_CUDA(cudaGetLastError());
+  return ATOS_OK;
+}
+
+// rank_out = x / n (R-PR-4) and the residual sum (conservation check) into *h_sum.
+int pr_finalize(Part& p, double* rank, const double* res, double* h_sum, cudaStream_t s) {
+  ATOS_TRY(p.scratch.ensure(64));
+  double* sum = p.scratch.as<double>();
+  ATOS_CUDA(cudaMemsetAsync(sum, 0, 8, s));
+  k_pr_finalize_n<<<148 * 8, 256, 0, s>>>(rank, res, p.n_local, (double)p.n_local, sum);
+  g_launches++;
+  ATOS_CUDA(cudaGetLastError());
+  ATOS_CUDA(cudaMemcpyAsync(h_sum, sum, 8, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  return ATOS_OK;
+}
+
 int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank, const Resolved& r,
                     atos_stats* st) {
   cudaStream_t s = r.stream;
