@@ -86,7 +86,8 @@ typedef struct {
     double   worker_ms;         /* device time of the worker kernel(s) alone (persistent launch, or the sum
                                    of the discrete launches incl. their host round trips), CUDA events */
     uint64_t timeline_len;      /* samples written to cfg->timeline */
-    uint64_t reserved[2];
+    uint64_t flags;             /* bit 0: BFS re-ran with the u32 depth state (depth >= 126 met) */
+    uint64_t reserved[1];
 } atos_stats;
 
 typedef struct {
@@ -121,7 +122,10 @@ typedef struct {
                                    workers every timeline_interval_ns -- the throughput-vs-time data of
                                    the paper's Figs. 1-3 */
     uint32_t timeline_interval_ns; /* 0 = 5000 */
-    int      reserved_i[3];
+    int      depth_state;       /* BFS state (dedupe mode): 0 = auto -- one byte per vertex (7-bit depth + queued
+                                   flag, L2-resident), re-run with u32 words if a depth >= 126 is met;
+                                   2 = u32 words from the start (high-diameter graphs) */
+    int      reserved_i[2];
 } atos_cfg;
 
 /* Fill *cfg with defaults (persistent, app-default worker/fetch, dedupe on). */

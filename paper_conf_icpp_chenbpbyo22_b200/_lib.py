@@ -37,7 +37,7 @@ class Stats(ctypes.Structure):
         ("pops", ctypes.c_uint64), ("pushes", ctypes.c_uint64), ("edges", ctypes.c_uint64),
         ("rounds", ctypes.c_uint64), ("bytes_exchanged", ctypes.c_uint64), ("kernel_ms", ctypes.c_double),
         ("residual_sum", ctypes.c_double), ("colors_used", ctypes.c_int64), ("worker_ms", ctypes.c_double),
-        ("timeline_len", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 2),
+        ("timeline_len", ctypes.c_uint64), ("flags", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 1),
     ]
 
     def as_dict(self):
@@ -53,7 +53,7 @@ class Cfg(ctypes.Structure):
         ("queue_capacity", ctypes.c_uint64), ("timeout_s", ctypes.c_double), ("stream", ctypes.c_void_p),
         ("stats", ctypes.POINTER(Stats)), ("l2_persist", ctypes.c_int), ("big_threshold", ctypes.c_int),
         ("big_chunk", ctypes.c_int), ("timeline_cap", ctypes.c_uint32), ("timeline", ctypes.c_void_p),
-        ("timeline_interval_ns", ctypes.c_uint32), ("reserved_i", ctypes.c_int * 3),
+        ("timeline_interval_ns", ctypes.c_uint32), ("depth_state", ctypes.c_int), ("reserved_i", ctypes.c_int * 2),
     ]
 
 

@@ -97,6 +97,11 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
   r->timeline_cap = d.timeline ? d.timeline_cap : 0;
   r->timeline_interval_ns = d.timeline_interval_ns ? d.timeline_interval_ns : 5000;
   r->big_threshold = d.big_threshold;
+  r->depth_state = d.depth_state;
+  if (r->depth_state != 0 && r->depth_state != 2) {
+    set_error("depth_state must be 0 (auto) or 2 (u32 words) (got %d)", r->depth_state);
+    return ATOS_ERR_INVALID_ARG;
+  }
   r->big_chunk = d.big_chunk;
   if (r->big_chunk < 0) {
     set_error("big_chunk must be >= 0");
@@ -243,6 +248,11 @@ int finish_queue(Part& p, cudaStream_t s, atos_stats* st, const char* what) {
     p.ring_clean = false;
     set_error("%s: device watchdog expired (no progress)", what);
     return ATOS_ERR_TIMEOUT;
+  }
+  if (status & kStatusDeep) {
+    // byte-state BFS stopped at an unencodable depth: the caller re-runs (the ring is reset then)
+    p.ring_clean = false;
+    return ATOS_OK;
   }
   if (h->done.v != h->tail.v) {
     p.ring_clean = false;

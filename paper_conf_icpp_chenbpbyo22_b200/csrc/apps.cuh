@@ -140,6 +140,76 @@ struct BfsAppT {
   }
 };
 
+// ------------------------------------------------------ BFS, byte state
+// Byte-state BFS: while depths stay below 126 the
+// whole per-vertex state is ONE byte -- bit 7 the queued flag, bits 0-6 the
+// depth, 126 = unreached -- so the state of a scale-26 graph is 67 MB and
+// stays in the 126 MB L2: the pop-time flag clear, the per-edge prefilter and
+// the improving CAS all hit L2 instead of a 268 MB u32 array in HBM.  Same
+// protocol as BfsAppT's dedupe mode (one CAS improves the depth and sets the
+// flag; the popper clears the flag with an acquire RMW that returns the
+// depth), on the aligned 32-bit word that holds the byte.  A pop at depth 125
+// cannot relax (126 is not encodable): it raises kStatusDeep and the host
+// re-runs the traversal with the u32 state (high-diameter graphs).
+constexpr uint32_t kBUnreached = 126u, kBMaxDepth = 125u, kBInq = 0x80u;
+
+struct BfsByteApp {
+  using Payload = uint32_t;  // d + 1
+  using Token = uint32_t;    // the 32-bit word holding w's state byte (prefilter and CAS guess)
+  const uint32_t* __restrict__ row_ptr;
+  const uint32_t* __restrict__ col;
+  uint8_t* state;            // n bytes, padded to a multiple of 4
+  uint32_t* status;          // queue control block status word
+  unsigned long long pol_first, pol_last;
+
+  __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
+  __device__ __forceinline__ void prepare() {
+    pol_first = policy_evict_first();
+    pol_last = policy_evict_last();
+  }
+  __device__ __forceinline__ uint32_t* word_of(uint32_t v) const { return (uint32_t*)(state + (v & ~3u)); }
+
+  __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
+    start = __ldg(row_ptr + v);
+    const uint32_t end = __ldg(row_ptr + v + 1);
+    const uint32_t sh = (v & 3u) * 8u;
+    const uint32_t d = (atom_and_acquire(word_of(v), ~(kBInq << sh)) >> sh) & 0x7Fu;
+    deg = end - start;
+    p = d + 1;
+    if (deg != 0 && d >= kBMaxDepth) {
+      atomicOr(status, kStatusDeep);
+      return false;
+    }
+    return deg != 0;
+  }
+  __device__ __forceinline__ Token pre(const Payload, uint32_t w) const {
+    uint32_t word;
+    asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(word) : "l"(word_of(w)), "l"(pol_last) : "memory");
+    return word;
+  }
+  // A stale word only over-states depths (they only decrease), so skipping on it is safe;
+  // the CAS decides everything else.
+  __device__ __forceinline__ bool post(const Payload nd, uint32_t w, Token word, uint32_t& out) const {
+    const uint32_t sh = (w & 3u) * 8u;
+    uint32_t* wp = word_of(w);
+    while (true) {
+      const uint32_t b = (word >> sh) & 0xFFu;
+      const uint32_t D = b & 0x7Fu;
+      if (D != kBUnreached && D <= nd) return false;
+      const uint32_t nw = (word & ~(0xFFu << sh)) | ((nd | kBInq) << sh);
+      const uint32_t old = atomicCAS(wp, word, nw);
+      if (old == word) {
+        out = w;
+        return !(b & kBInq);  // queue w unless it is already queued (dedupe)
+      }
+      word = old;
+    }
+  }
+  __device__ __forceinline__ bool relax(const Payload nd, uint32_t w, uint32_t& out) const {
+    return post(nd, w, pre(nd, w), out);
+  }
+};
+
 // -------------------------------------------------------------- PageRank
 // Asynchronous push PageRank relax (Alg.4):
 //   res = atomicExch(residue+v, 0); atomicAdd(rank+v, res);

@@ -33,6 +33,7 @@ constexpr uint32_t kUnreached = 0xFFFFFFFFu;
 // status bits written by the device watchdog
 constexpr uint32_t kStatusOverflow = 1u;
 constexpr uint32_t kStatusTimeout = 2u;
+constexpr uint32_t kStatusDeep = 4u;     // byte-state BFS met a depth it cannot encode (host re-runs)
 
 struct __align__(128) Line64 {
   unsigned long long v;

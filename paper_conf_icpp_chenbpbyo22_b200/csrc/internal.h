@@ -112,7 +112,7 @@ struct DeviceGuard {
 
 struct Resolved {
   int persistent, worker, fetch, num_blocks, block_threads, dedupe, check_size;
-  int conflict_policy, permute_init, validate, out_where, l2_persist, big_threshold, big_chunk;
+  int conflict_policy, permute_init, validate, out_where, l2_persist, big_threshold, big_chunk, depth_state;
   unsigned long long* timeline;
   uint32_t timeline_cap, timeline_interval_ns;
   uint64_t queue_capacity;

@@ -55,6 +55,33 @@ __global__ void k_bfs_init(uint32_t* depth, int dedupe, uint8_t* shadow, Ring q,
   }
 }
 
+// Byte-state BFS init: state[] was memset to kBUnreached; source depth 0, queued.
+__global__ void k_bfs_byte_init(uint8_t* state, Ring q, uint32_t src, unsigned long long wd) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    run_begin(q.ctl);
+    state[src] = (uint8_t)kBInq;
+    const unsigned long long idx = q.ctl->tail.v;
+    q.ctl->tail.v = idx + 1;
+    publish_one(q, idx, src, wd);
+  }
+}
+
+// depth_out from the byte state (kBUnreached -> 0xFFFFFFFF), 4 vertices per thread.
+__global__ void k_bfs_byte_output(const uint8_t* __restrict__ state, uint32_t* depth, int64_t n) {
+  const int64_t nw = (n + 3) / 4;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nw; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t word = ((const uint32_t*)state)[i];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int64_t v = 4 * i + k;
+      if (v < n) {
+        const uint32_t D = (word >> (8 * k)) & 0x7Fu;
+        depth[v] = D == kBUnreached ? 0xFFFFFFFFu : D;
+      }
+    }
+  }
+}
+
 // PageRank vertex init (Alg.3): rank = 1 - lambda, residue = 0.
 __global__ void k_pr_init_vertices(double* rank, double* res, int64_t n, double one_minus_alpha) {
   for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
@@ -275,12 +302,54 @@ static Ring ring_of(Part& p) {
 }
 
 // --------------------------------------------------------------------- BFS
+// Byte-state traversal (BfsByteApp).  *deep = true when a depth >= 126 was met
+// (nothing is written to depth then; the caller re-runs with the u32 state).
+static int bfs_single_bytes(Part& p, int64_t src, uint32_t* depth, const Resolved& r, atos_stats* st, bool* deep) {
+  cudaStream_t s = r.stream;
+  const int64_t n = p.n_local;
+  *deep = false;
+  const size_t nb = (size_t)(n + 3) / 4 * 4;
+  ATOS_TRY(p.shadow.ensure(nb));
+  uint8_t* state = p.shadow.as<uint8_t>();
+  ATOS_CUDA(cudaMemsetAsync(state, (int)kBUnreached, nb, s));
+  Ring q = ring_of(p);
+  k_bfs_byte_init<<<1, 32, 0, s>>>(state, q, (uint32_t)src, r.watchdog_ns);
+  g_launches++;
+  ATOS_CUDA(cudaGetLastError());
+  if (r.l2_persist) set_l2_window(s, state, nb, true);
+  BfsByteApp app{p.row_ptr, p.col, state, (uint32_t*)&q.ctl->status.v, 0ull, 0ull};
+  p.ring_clean = false;
+  int rc = launch_relax(app, q, r, p, st);
+  if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
+  if (rc != ATOS_OK) return rc;
+  ATOS_TRY(finish_queue(p, s, st, "bfs"));
+  if (((QueueCtl*)p.host_pinned)->status.v & kStatusDeep) {
+    *deep = true;
+    return ATOS_OK;
+  }
+  k_bfs_byte_output<<<148 * 8, 256, 0, s>>>(state, depth, n);
+  g_launches++;
+  ATOS_CUDA(cudaGetLastError());
+  return ATOS_OK;
+}
+
 int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolved& r, atos_stats* st) {
   cudaStream_t s = r.stream;
   const int64_t n = p.n_local;
   uint64_t want = r.queue_capacity ? r.queue_capacity : (uint64_t)std::max<int64_t>(2 * n, 1024);
   if (!r.dedupe && !r.queue_capacity) want = (uint64_t)std::max<int64_t>(4 * n, 4096);
   ATOS_TRY(ensure_queue(p, pow2_at_least(want), s));
+  // byte state first (dedupe mode); a traversal deeper than 125 levels re-runs with u32 words
+  if (r.dedupe && r.depth_state != 2) {
+    bool deep = false;
+    ATOS_TRY(bfs_single_bytes(p, src, depth, r, st, &deep));
+    if (!deep) return ATOS_OK;
+    if (st) {
+      st->flags |= 1;  // re-run with the u32 state; rounds describe the final run (worker_ms keeps both)
+      st->rounds = 0;
+    }
+    ATOS_TRY(ensure_queue(p, pow2_at_least(want), s));  // resets the ring the stopped run left behind
+  }
   ATOS_CUDA(cudaMemsetAsync(depth, 0xFF, (size_t)n * 4, s));
   ATOS_TRY(p.shadow.ensure((size_t)n));
   uint8_t* shadow = p.shadow.as<uint8_t>();

@@ -37,6 +37,10 @@ KNOBS = [
     dict(worker=32, fetch_size=8, big_threshold=32, big_chunk=8),
     dict(worker=128, fetch_size=32, big_threshold=8, big_chunk=1, dedupe=0),
     dict(worker=256, fetch_size=256, big_threshold=-1),
+    # the u32 depth-word state (the byte state's fallback for depths >= 126) forced from the start
+    dict(worker=256, fetch_size=256, depth_state=2),
+    dict(worker=32, fetch_size=8, depth_state=2),
+    dict(worker=1, fetch_size=2, persistent=0, depth_state=2),
 ]
 
 
@@ -170,3 +174,31 @@ def test_config_c1_bench_launch():
     for knobs in (dict(), dict(worker=32), dict(persistent=0)):
         d, st = atos.bfs(csr, src, **knobs)
         np.testing.assert_array_equal(as_u32(d), want)
+
+
+@pytest.mark.parametrize("n,deep", [(125, False), (126, True), (400, True)])
+def test_byte_state_depth_boundary(n, deep):
+    """Byte state encodes depths 0..125; a pop at depth 125 with edges re-runs with u32 words
+    (stats flag bit 0).  Results are bit-exact either way."""
+    rp, ci = G.path(n)
+    csr = csr_of(rp, ci)
+    want = oracle.bfs(rp, ci, 0)
+    for knobs in (dict(), dict(worker=32, fetch_size=4), dict(persistent=0)):
+        d, st = atos.bfs(csr, 0, **knobs)
+        np.testing.assert_array_equal(as_u32(d), want)
+        assert bool(st["flags"] & 1) == deep
+        d2, st2 = atos.bfs(csr, 0, depth_state=2, **knobs)
+        np.testing.assert_array_equal(as_u32(d2), want)
+        assert st2["flags"] == 0
+
+
+def test_byte_state_word_neighbours():
+    """Four consecutive vertex ids share one 32-bit state word: a 4-clique plus pendant chains
+    exercises CAS retries on neighbouring bytes."""
+    edges = [(a, b) for a in range(4) for b in range(4) if a != b]
+    edges += [(k, 4 + k) for k in range(4)] + [(4 + k, 8 + k) for k in range(4)]
+    rp, ci = G.csr_from_edges(12, edges, symmetric=True)
+    csr = csr_of(rp, ci)
+    for src in range(12):
+        d, _ = atos.bfs(csr, src)
+        np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, src))
