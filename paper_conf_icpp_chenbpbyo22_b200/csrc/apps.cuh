@@ -47,6 +47,7 @@ struct GhostView {
 // partition, where every neighbour is local and vb == 0.
 template <bool PART>
 struct BfsAppT {
+  static constexpr bool kAcquirePop = true;  // paper-literal mode reads depth[v] with a plain load
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
   const uint32_t* __restrict__ row_ptr;
@@ -154,6 +155,7 @@ struct BfsAppT {
 constexpr uint32_t kBUnreached = 126u, kBMaxDepth = 125u, kBInq = 0x80u;
 
 struct BfsByteApp {
+  static constexpr bool kAcquirePop = false;  // the popper reads the state only through its RMW
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // the 32-bit word holding w's state byte (prefilter and CAS guess)
   const uint32_t* __restrict__ row_ptr;
@@ -173,7 +175,9 @@ struct BfsByteApp {
     start = __ldg(row_ptr + v);
     const uint32_t end = __ldg(row_ptr + v + 1);
     const uint32_t sh = (v & 3u) * 8u;
-    const uint32_t d = (atom_and_acquire(word_of(v), ~(kBInq << sh)) >> sh) & 0x7Fu;
+    // relaxed: the RMW returns the latest depth in coherence order, and nothing else the
+    // pusher wrote is read (no acquire, so no L1 invalidation per pop)
+    const uint32_t d = (atomicAnd(word_of(v), ~(kBInq << sh)) >> sh) & 0x7Fu;
     deg = end - start;
     p = d + 1;
     if (deg != 0 && d >= kBMaxDepth) {
@@ -219,6 +223,7 @@ struct BfsByteApp {
 // atomic), which keeps "residue[v] > eps  =>  v queued or in flight".
 template <bool PART>
 struct PrAppT {
+  static constexpr bool kAcquirePop = false;  // residue taken with atomicExch (RMW)
   using Payload = double;  // delta = alpha * rho / deg(v)
   using Token = double;    // residue before our atomicAdd
   const uint32_t* __restrict__ row_ptr;

@@ -240,14 +240,22 @@ __device__ __forceinline__ void publish_one(const Ring& q, unsigned long long id
 // Try to take the item of index idx: 1 = taken (*item set, slot freed for the
 // next lap), 0 = not published yet, -1 = the item was stolen by a lap-blocked
 // producer (drop the claim).
+// ACQ = false (apps whose per-item state is only touched through RMWs, e.g. the
+// BFS state word and the PageRank residue): relaxed load and CAS -- no L1
+// invalidation (CCTL.IVALL) or MEMBAR per consumed item.  The item id itself is
+// the only payload; everything the consumer then reads about the vertex comes
+// from an atomic RMW, which always observes the latest value in coherence order.
+template <bool ACQ = true>
 __device__ __forceinline__ int try_consume(const Ring& q, unsigned long long idx, uint32_t* item) {
   unsigned long long* slot = q.slots + (idx & q.mask);
   unsigned long long v;
-  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(slot) : "memory");
+  if (ACQ) asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(slot) : "memory");
+  else asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(slot) : "memory");
   const int32_t d = (int32_t)((uint32_t)(v >> 32) - (uint32_t)(idx + 1));
   if (d < 0) return 0;
   if (d > 0) return -1;
-  if (atom_cas_acq_rel(slot, v, make_slot(idx + q.mask + 1, 0u)) != v) return -1;
+  const unsigned long long freed = make_slot(idx + q.mask + 1, 0u);
+  if ((ACQ ? atom_cas_acq_rel(slot, v, freed) : atomicCAS(slot, v, freed)) != v) return -1;
   *item = (uint32_t)v;
   return 1;
 }

@@ -291,11 +291,11 @@ __device__ __forceinline__ uint32_t group_size() {
 
 // Try to consume index `idx`: on success the item goes to s.item[] (slot freed
 // for the next lap); otherwise idx is appended to the new pending list.
-template <class Payload>
+template <bool ACQ, class Payload>
 __device__ __forceinline__ void consume_slot(const Ring& q, const GroupSmem<Payload>& s,
                                              unsigned long long idx) {
   uint32_t v;
-  const int rc = try_consume(q, idx, &v);
+  const int rc = try_consume<ACQ>(q, idx, &v);
   if (rc == 0) {
     uint32_t k = atomicAdd(&s.ctr[2], 1u);
     s.pend2[k] = idx;
@@ -309,7 +309,7 @@ __device__ __forceinline__ void consume_slot(const Ring& q, const GroupSmem<Payl
 // One worker (a CTA, a warp, or -- for MODE_THREAD -- a warp of 32 thread
 // workers that share one claim) and its queue protocol: claim / gather /
 // idle-with-termination (acquire) and completion (complete).
-template <int MODE, bool PERSIST, class Payload>
+template <int MODE, bool PERSIST, class Payload, bool ACQ = true>
 struct Worker {
   GroupSmem<Payload> s;
   uint32_t r, G, K;
@@ -393,8 +393,8 @@ struct Worker {
       {
         const unsigned long long cb = *(unsigned long long*)&s.ctr[6];
         const uint32_t cc = s.ctr[4], np = s.ctr[1];
-        for (uint32_t i = r; i < cc; i += G) consume_slot(q, s, cb + i);
-        for (uint32_t i = r; i < np; i += G) consume_slot(q, s, s.pend[i]);
+        for (uint32_t i = r; i < cc; i += G) consume_slot<ACQ>(q, s, cb + i);
+        for (uint32_t i = r; i < np; i += G) consume_slot<ACQ>(q, s, s.pend[i]);
       }
       group_sync<MODE>();
       const uint32_t nready = s.ctr[0];
@@ -474,7 +474,7 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
   const uint32_t nwarps = blockDim.x >> 5;
   // push rings first (kPushBuf u32 per warp), then one arena per group
   uint32_t* pushbuf = (uint32_t*)smem_raw;
-  Worker<MODE, PERSIST, Payload> wk;
+  Worker<MODE, PERSIST, Payload, App::kAcquirePop> wk;
   wk.init(smem_raw + (size_t)nwarps * kPushBuf * 4, P);
   const GroupSmem<Payload>& s = wk.s;
   const uint32_t r = wk.r, G = wk.G;
