@@ -52,6 +52,14 @@ def measured_peaks():
     return 6650.0, "fallback"
 
 
+def micro_peak(key: str):
+    """Access-pattern ceilings measured by tools/micro (profiles/r01_micro_peaks.json)."""
+    p = os.path.join(ROOT, "profiles", "r01_micro_peaks.json")
+    if os.path.exists(p):
+        return float(json.load(open(p))[key]["value"])
+    return None
+
+
 def profile_traffic(kernel_key: str):
     """dram bytes per launch from the committed ncu --set full summary (profiles/), or None."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
@@ -263,6 +271,13 @@ def run_atos(args, ws, rank, local):
                 "traffic": profile_traffic("bfs_worker"), "peak_kind": peak_kind,
                 "kernel": "k_relax_worker<BfsApp,CTA,persistent>", "kernel_ms": w_ms,
                 "worker_share_of_step": w_ms / ms_per_step}
+    gpk = micro_peak("random_gather_per_s")
+    if gpk:
+        # the per-edge state gather is one uncoalesced L1TEX wavefront: the access pattern's own ceiling
+        ach = np.mean(edges) / ws / (w_ms / 1e3)
+        roofline["pattern_roofline"] = {"bound": "l1tex random-gather wavefronts (1 per edge)", "achieved": ach,
+                                        "peak": gpk, "unit": "edges/s", "frac": ach / gpk,
+                                        "peak_source": "profiles/r01_micro_peaks.json"}
     line = {
         "metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak" if ws == 1 else "strong",
@@ -384,6 +399,12 @@ def run_apps(args, dev, peak):
                        "pops_per_n": float(np.mean(pops)) / g.n, "edge_relaxations_per_m": float(np.mean(edges)) / g.m,
                        "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
                        "traffic": profile_traffic("pr_worker")}
+    apk = micro_peak("l2_atomic_add_with_return_per_s")
+    if apk:
+        ach = float(np.mean(edges)) / (wm / 1e3)
+        res["pagerank"]["pattern_roofline"] = {"bound": "L2 atomic add with return (1 per edge relaxation)",
+                                               "achieved": ach, "peak": apk, "unit": "atomics/s", "frac": ach / apk,
+                                               "peak_source": "profiles/r01_micro_peaks.json"}
     if not args.no_bsp:
         res["pagerank"]["bsp"] = bsp_app(lambda: atos.pagerank_bsp(csr, 0.85, 1e-6, out=out), flush, g,
                                          float(np.mean(ms)))

@@ -103,8 +103,10 @@ typedef struct {
                                    0: paper-literal push on every improvement */
     int      check_size;        /* PageRank: 0 = threshold-crossing activation (default);
                                    >0 = the paper's round-robin Check_Size sweep */
-    int      conflict_policy;   /* colouring: 0 = the lower-priority endpoint is recoloured (default);
-                                   1 = paper-literal, the checker re-queues itself */
+    int      conflict_policy;   /* colouring: 0 = the lower-priority endpoint is recoloured (default;
+                                   priority = degree, then splitmix64(seed ^ v), then id);
+                                   1 = paper-literal, the checker re-queues itself;
+                                   2 = as 0 with the hash priority only (no degree term) */
     int      permute_init;      /* colouring: 1 = seed-permuted initial queue order; 0 = vertex-ID order */
     int      validate;          /* 1: check CSR invariants / symmetry at call time (O(m)) */
     int      out_where;         /* ATOS_MEM_DEVICE (default) or ATOS_MEM_HOST for the output buffer */
@@ -193,7 +195,7 @@ ATOS_API int atos_color(const atos_csr* g, uint64_t seed, int32_t* color_out, co
  *                       scale and error bound as atos_pagerank.
  *  - atos_color_bsp:    Alg.5: assign kernel, barrier, conflict
  *                       kernel; a conflict re-queues the lower-priority
- *                       endpoint (priority splitmix64(seed ^ v)), or both
+ *                       endpoint (priority as atos_color), or both
  *                       endpoints with cfg->conflict_policy = 1 (the literal
  *                       Alg.5, which may not terminate: set timeout_s).
  * Used cfg fields: stream, stats, out_where, timeout_s, validate

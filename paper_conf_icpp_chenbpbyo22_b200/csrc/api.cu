@@ -85,6 +85,10 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
     return ATOS_ERR_INVALID_ARG;
   }
   r->conflict_policy = d.conflict_policy;
+  if (r->conflict_policy < 0 || r->conflict_policy > 2) {
+    set_error("conflict_policy must be 0, 1 or 2 (got %d)", r->conflict_policy);
+    return ATOS_ERR_INVALID_ARG;
+  }
   r->permute_init = d.permute_init;
   r->validate = d.validate;
   r->out_where = d.out_where;

@@ -13,8 +13,8 @@
 //                       as R-GC-4) then, after a barrier, a conflict kernel
 //                       whose conflicting vertices form the next frontier.
 //                       Alg.5 appends BOTH endpoints of a conflict; read as
-//                       R-GC-2 (the lower-priority endpoint, priority
-//                       splitmix64(seed ^ v)), literal policy as the knob
+//                       R-GC-2 (the lower-priority endpoint, priority = degree,
+//                       then splitmix64(seed ^ v)), literal policy as the knob
 //                       conflict_policy = 1 (may livelock; honours timeout_s).
 // The barrier is the host round trip of the paper's cudaDeviceSynchronize()
 // (the frontier size is read back every iteration).
@@ -202,7 +202,15 @@ __global__ void k_bsp_pr_filter(const double* __restrict__ res, uint32_t n, doub
 }
 
 // ------------------------------------------------------------------ colouring
-__device__ __forceinline__ bool bsp_loses(unsigned long long seed, uint32_t x, uint32_t y) {
+// R-GC-2, as the asynchronous path: lower degree loses, then lower hash priority, then lower id
+// (policy 2: hash priority only)
+__device__ __forceinline__ bool bsp_loses(const uint32_t* __restrict__ row_ptr, int hash_only,
+                                          unsigned long long seed, uint32_t x, uint32_t y) {
+  if (!hash_only) {
+    const uint32_t dx = __ldg(row_ptr + x + 1) - __ldg(row_ptr + x);
+    const uint32_t dy = __ldg(row_ptr + y + 1) - __ldg(row_ptr + y);
+    if (dx != dy) return dx < dy;
+  }
   const unsigned long long px = splitmix64(seed ^ x), py = splitmix64(seed ^ y);
   return px < py || (px == py && x < y);
 }
@@ -261,7 +269,7 @@ __global__ void __launch_bounds__(256) k_bsp_color_conflicts(const uint32_t* __r
                                                              const uint32_t* __restrict__ col,
                                                              const int32_t* __restrict__ color,
                                                              const uint32_t* __restrict__ front, uint32_t F,
-                                                             unsigned long long seed, int literal, uint32_t* out,
+                                                             unsigned long long seed, int literal /* conflict_policy */, uint32_t* out,
                                                              unsigned long long* nout, unsigned long long* reset,
                                                              unsigned long long* edges) {
   if (blockIdx.x == 0 && threadIdx.x == 0) *reset = 0;
@@ -274,7 +282,7 @@ __global__ void __launch_bounds__(256) k_bsp_color_conflicts(const uint32_t* __r
     bool bad = false;
     for (uint32_t j = lane; j < deg && !bad; j += 32) {
       const uint32_t w = __ldg(col + st + j);
-      if (w != v && color[w] == cv && (literal || bsp_loses(seed, v, w))) bad = true;
+      if (w != v && color[w] == cv && (literal == 1 || bsp_loses(row_ptr, literal == 2, seed, v, w))) bad = true;
     }
     const bool any = __ballot_sync(0xffffffffu, bad) != 0;
     if (lane == 0) {
@@ -456,7 +464,7 @@ int color_bsp_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const 
     k_bsp_color_assign<<<grid, 256, 0, s>>>(p.row_ptr, p.col, color, b.fa, (uint32_t)F, b.ctr + 1);
     // barrier, then conflict detection
     k_bsp_color_conflicts<<<grid, 256, 0, s>>>(p.row_ptr, p.col, color, b.fa, (uint32_t)F, seed,
-                                                r.conflict_policy == 1 ? 1 : 0, b.fb, cnt,
+                                                r.conflict_policy, b.fb, cnt,
                                                 b.ctr + 2 * ((it + 1) & 1), b.ctr + 1);
     g_launches += 2;
     ATOS_CUDA(cudaGetLastError());

@@ -31,9 +31,19 @@ struct ColorCtx {
   uint32_t* inq;            // assign-task dedupe bitmap (always on for colouring)
   unsigned long long seed;
   int literal;              // 1: paper-literal self-recolour policy
+  int hash_only;            // 1: conflict priority by hash only (conflict_policy 2)
 
-  // true when x loses against y: lower priority (splitmix64(seed ^ id), then id)
+  // true when x loses against y (R-GC-2): by default the lower-DEGREE endpoint
+  // recolours (largest-degree-first, so hubs -- whose assign tasks cost a
+  // whole neighbour scan -- are not recoloured for every low-degree neighbour
+  // they collide with), then lower priority splitmix64(seed ^ id), then id.
+  // conflict_policy 2: hash priority only.
   __device__ __forceinline__ bool loses(uint32_t x, uint32_t y) const {
+    if (!hash_only) {
+      const uint32_t dx = __ldg(row_ptr + x + 1) - __ldg(row_ptr + x);
+      const uint32_t dy = __ldg(row_ptr + y + 1) - __ldg(row_ptr + y);
+      if (dx != dy) return dx < dy;
+    }
     const unsigned long long px = splitmix64(seed ^ x), py = splitmix64(seed ^ y);
     return px < py || (px == py && x < y);
   }
@@ -544,7 +554,8 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   q.slots = p.ring.as<unsigned long long>();
   q.mask = p.ring_cap - 1;
   q.ctl = p.ctl.as<QueueCtl>();
-  ColorCtx c{p.row_ptr, p.col, color, p.bitmap.as<uint32_t>(), seed, r.conflict_policy == 1 ? 1 : 0};
+  ColorCtx c{p.row_ptr, p.col, color, p.bitmap.as<uint32_t>(), seed, r.conflict_policy == 1 ? 1 : 0,
+             r.conflict_policy == 2 ? 1 : 0};
   // init: reserve [t, t+n) then publish every vertex
   k_color_begin<<<1, 32, 0, s>>>(q.ctl, n);
   g_launches++;
