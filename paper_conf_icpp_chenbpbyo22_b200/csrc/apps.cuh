@@ -45,9 +45,11 @@ struct GhostView {
 
 // PART (compile time): partitioned run (ghosts, local ids); false = single
 // partition, where every neighbour is local and vb == 0.
-template <bool PART>
+// ACQ: acquire pops.  Needed only by the paper-literal mode (dedupe = 0), which
+// reads depth[v] with a plain load; the dedupe mode reads it through its RMW.
+template <bool PART, bool ACQ = true>
 struct BfsAppT {
-  static constexpr bool kAcquirePop = true;  // paper-literal mode reads depth[v] with a plain load
+  static constexpr bool kAcquirePop = ACQ;
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
   const uint32_t* __restrict__ row_ptr;
@@ -69,7 +71,7 @@ struct BfsAppT {
     start = __ldg(row_ptr + v);
     const uint32_t end = __ldg(row_ptr + v + 1);
     uint32_t d;
-    if (dedupe) d = atom_and_acquire(depth + v, ~kInq) & kDepthMask;
+    if (dedupe) d = (ACQ ? atom_and_acquire(depth + v, ~kInq) : atomicAnd(depth + v, ~kInq)) & kDepthMask;
     else d = ld_relaxed(depth + v);  // coherent read (L2): the value that caused the push
     deg = end - start;
     p = d + 1;
@@ -280,6 +282,7 @@ struct PrAppT {
 };
 
 using BfsApp = BfsAppT<false>;
+using BfsDedupeApp = BfsAppT<false, false>;  // u32 state, dedupe mode: relaxed pops
 using BfsPartApp = BfsAppT<true>;
 using PrApp = PrAppT<false>;
 using PrPartApp = PrAppT<true>;

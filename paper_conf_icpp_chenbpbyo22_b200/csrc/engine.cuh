@@ -41,6 +41,9 @@ constexpr uint32_t kCown = 2048;  // CTA mode: per-batch owner table of 32*kU-ed
 #ifndef ATOS_MINB
 #define ATOS_MINB 1
 #endif
+#ifndef ATOS_BACKOFF_MAX
+#define ATOS_BACKOFF_MAX 1024  // idle poll backoff cap (ns)
+#endif
 
 // ------------------------------------------------------------ big-task assist
 // A popped vertex whose degree exceeds big_threshold is not expanded by the
@@ -428,7 +431,7 @@ struct Worker {
           }
           tl_sample(P);
           __nanosleep(backoff);
-          backoff = backoff < 1024 ? backoff * 2 : 1024;
+          backoff = backoff < ATOS_BACKOFF_MAX ? backoff * 2 : ATOS_BACKOFF_MAX;
         }
       }
       group_sync<MODE>();

@@ -359,9 +359,11 @@ int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolve
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, depth, (size_t)n * 4, true);
-  BfsApp app{p.row_ptr, p.col, depth, r.dedupe, shadow, 0ull, 0ull, GhostView{0u, (uint32_t)n, nullptr, nullptr, nullptr}};
+  const GhostView nogv{0u, (uint32_t)n, nullptr, nullptr, nullptr};
   p.ring_clean = false;
-  int rc = launch_relax(app, q, r, p, st);
+  int rc;
+  if (r.dedupe) rc = launch_relax(BfsDedupeApp{p.row_ptr, p.col, depth, 1, shadow, 0ull, 0ull, nogv}, q, r, p, st);
+  else rc = launch_relax(BfsApp{p.row_ptr, p.col, depth, 0, shadow, 0ull, 0ull, nogv}, q, r, p, st);
   if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
   if (rc != ATOS_OK) return rc;
   return finish_queue(p, s, st, "bfs");
