@@ -41,6 +41,10 @@ constexpr uint32_t kCown = 2048;  // CTA mode: per-batch owner table of 32*kU-ed
 #ifndef ATOS_MINB
 #define ATOS_MINB 1
 #endif
+#ifndef ATOS_MIN_CLAIM
+#define ATOS_MIN_CLAIM 16
+#endif
+constexpr unsigned long long kMinClaim = ATOS_MIN_CLAIM;  // smallest fair-share claim (items)
 #ifndef ATOS_BACKOFF_MAX
 #define ATOS_BACKOFF_MAX 1024  // idle poll backoff cap (ns)
 #endif
@@ -367,16 +371,25 @@ struct Worker {
           // Sparse queue: an exact CAS claim of what is visible, so no index past
           // the tail is ever parked in a sleeping worker's pending list (that made
           // late improvement cascades crawl one backoff period per item).
+          // Claim size: K, or -- when the visible work is thin relative to the
+          // number of workers (a high-diameter frontier) -- the fair share
+          // visible / workers, at least kMinClaim, so one worker does not
+          // serialise a whole small frontier while the others idle.
           unsigned long long h = ld_relaxed(&q.ctl->head.v);
           const unsigned long long t = ld_relaxed(&q.ctl->tail.v);
           if (h < t) {
-            if (t - h >= 2ull * K) {
-              const unsigned long long b = atomicAdd(&q.ctl->head.v, (unsigned long long)K);
+            const unsigned long long nworkers =
+                (unsigned long long)gridDim.x * (MODE == MODE_CTA ? 1u : (blockDim.x >> 5));
+            unsigned long long want = (t - h) / nworkers;
+            const unsigned long long lo = K < kMinClaim ? K : kMinClaim;
+            want = want < lo ? lo : (want > K ? K : want);
+            if (t - h >= 2ull * want) {
+              const unsigned long long b = atomicAdd(&q.ctl->head.v, want);
               *(unsigned long long*)&s.ctr[6] = b;
-              s.ctr[4] = K;
+              s.ctr[4] = (uint32_t)want;
             } else {
               for (int tries = 0; tries < 4 && h < t; ++tries) {
-                const unsigned long long amt = t - h < K ? t - h : K;
+                const unsigned long long amt = t - h < want ? t - h : want;
                 const unsigned long long old = atomicCAS(&q.ctl->head.v, h, h + amt);
                 if (old == h) {
                   *(unsigned long long*)&s.ctr[6] = h;
