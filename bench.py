@@ -269,7 +269,7 @@ def run_atos(args, ws, rank, local):
     achieved = alg_bytes / (w_ms / 1e3) / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": profile_traffic("bfs_worker"), "peak_kind": peak_kind,
-                "kernel": "k_relax_worker<BfsApp,CTA,persistent>", "kernel_ms": w_ms,
+                "kernel": "k_relax_worker<BfsByteApp,CTA,persistent>", "kernel_ms": w_ms,
                 "worker_share_of_step": w_ms / ms_per_step}
     gpk = micro_peak("random_gather_per_s")
     if gpk:
