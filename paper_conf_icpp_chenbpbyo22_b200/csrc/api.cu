@@ -319,14 +319,27 @@ static int upload_part(Part& p, int64_t n_global, const int64_t* row_ptr, const 
   if (where == ATOS_MEM_HOST) {
     // upload the int64 offsets as they are and narrow on the device (a host loop over n
     // would cost more than the copy); col goes straight into its final buffer
+    // (whole-graph uploads are also validated there: monotone, 0 .. m -- see validate_host_csr)
     int64_t* tmp = nullptr;
-    ATOS_CUDA(cudaMalloc(&tmp, (size_t)(nl + 1) * 8));
+    unsigned* bad = nullptr;
+    ATOS_CUDA(cudaMalloc(&tmp, (size_t)(nl + 1) * 8 + 16));
+    bad = (unsigned*)(tmp + nl + 1);
+    ATOS_CUDA(cudaMemset(bad, 0, 4));
     ATOS_CUDA(cudaMemcpy(tmp, row_ptr + v_begin, (size_t)(nl + 1) * 8, cudaMemcpyHostToDevice));
-    k_rebase_row_ptr<<<1024, 256>>>(tmp, p.row_ptr, nl + 1, e_begin);
+    if (v_begin == 0 && v_end == n_global) {
+      k_narrow_row_ptr<<<1024, 256>>>(tmp, p.row_ptr, nl + 1, ml, bad);
+    } else {
+      k_rebase_row_ptr<<<1024, 256>>>(tmp, p.row_ptr, nl + 1, e_begin);
+    }
     g_launches++;
     if (ml) ATOS_CUDA(cudaMemcpy(p.col, col + e_begin, (size_t)ml * 4, cudaMemcpyHostToDevice));
-    ATOS_CUDA(cudaDeviceSynchronize());
+    unsigned hb = 0;
+    ATOS_CUDA(cudaMemcpy(&hb, bad, 4, cudaMemcpyDeviceToHost));
     cudaFree(tmp);
+    if (hb) {
+      set_error("row_ptr is not non-decreasing (or outside [0, m])");
+      return ATOS_ERR_INVALID_ARG;
+    }
     return ATOS_OK;
   }
   // device input: rebase + narrow on the device
@@ -363,18 +376,21 @@ int upload_part_local(Part& p, const int64_t* row_ptr, const int32_t* col, int w
   return ATOS_OK;
 }
 
-// host CSR: offsets checked on the host (O(n)); col ids are checked on the device
-// after the upload (validate_uploaded_cols), which is far cheaper than a host pass over m
-static int validate_host_csr(int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col) {
+// host CSR: the end points are checked here; monotonicity while the offsets are
+// narrowed on the device (single partition: k_narrow_row_ptr in upload_part; loopback
+// partitions: the host loop below) and col ids after the upload
+// (validate_uploaded_cols) -- a host pass over n or m would cost more than the copy
+static int validate_host_csr(int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col, bool full) {
   if (row_ptr[0] != 0 || row_ptr[n] != m) {
     set_error("row_ptr[0] must be 0 and row_ptr[n] must equal m");
     return ATOS_ERR_INVALID_ARG;
   }
-  for (int64_t v = 0; v < n; ++v)
-    if (row_ptr[v + 1] < row_ptr[v]) {
-      set_error("row_ptr is not non-decreasing at %lld", (long long)v);
-      return ATOS_ERR_INVALID_ARG;
-    }
+  if (full)
+    for (int64_t v = 0; v < n; ++v)
+      if (row_ptr[v + 1] < row_ptr[v]) {
+        set_error("row_ptr is not non-decreasing at %lld", (long long)v);
+        return ATOS_ERR_INVALID_ARG;
+      }
   (void)col;
   return ATOS_OK;
 }
@@ -519,7 +535,8 @@ int atos_csr_create(atos_csr** out, int64_t n, int64_t m, const int64_t* row_ptr
   }
   DeviceGuard dg(device);
   if (n > 0) {
-    int rc = where == ATOS_MEM_HOST ? validate_host_csr(n, m, row_ptr, col) : validate_device_csr(n, m, row_ptr, col);
+    int rc = where == ATOS_MEM_HOST ? validate_host_csr(n, m, row_ptr, col, num_parts > 1)
+                                    : validate_device_csr(n, m, row_ptr, col);
     if (rc != ATOS_OK) return rc;
   }
   atos_csr* g = new atos_csr();

@@ -147,6 +147,22 @@ def test_errors():
         atos.CSR(bad_rp, torch.tensor([1, 0], dtype=torch.int32, device=DEV))
     with pytest.raises(RuntimeError, match="INVALID_ARG"):
         atos.CSR(torch.tensor([0, 1], dtype=torch.int64), torch.tensor([5], dtype=torch.int32))
+    # host input: non-monotone offsets are caught while narrowing on the device, for one
+    # partition and for loopback partitions (host check)
+    bad_h = torch.tensor([0, 2, 1, 3], dtype=torch.int64)
+    cols_h = torch.tensor([1, 2, 0], dtype=torch.int32)
+    for parts in (1, 2):
+        with pytest.raises(RuntimeError, match="INVALID_ARG"):
+            atos.CSR(bad_h, cols_h, num_parts=parts)
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.CSR(torch.tensor([0, 1, 3, 2], dtype=torch.int64), cols_h)  # row_ptr[n] != m
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.CSR(torch.tensor([0, 4, 2, 3], dtype=torch.int64), cols_h)  # offset > m inside
+    # rejected at conflict_policy outside 0..2 and depth_state outside {0, 2}
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.color(csr, 1, conflict_policy=3)
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.bfs(csr, 0, depth_state=1)
 
 
 def test_small_queue_overflow_reports_error():

@@ -26,6 +26,8 @@ KNOBS = [
     dict(worker=1, fetch_size=1, persistent=0),
     dict(worker=32, fetch_size=8, permute_init=1),
     dict(worker=256, fetch_size=128, permute_init=1),
+    dict(worker=1024, fetch_size=128, conflict_policy=2),  # hash-only priority
+    dict(worker=32, fetch_size=8, conflict_policy=2),
 ]
 
 
