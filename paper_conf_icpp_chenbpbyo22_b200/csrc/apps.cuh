@@ -157,7 +157,10 @@ struct BfsAppT {
 constexpr uint32_t kBUnreached = 126u, kBMaxDepth = 125u, kBInq = 0x80u;
 
 struct BfsByteApp {
-  static constexpr bool kAcquirePop = false;  // the popper reads the state only through its RMW
+  // Acquire pops: the slot load must synchronise with the pusher's release so that the
+  // popper's AND is ordered after the pusher's CAS on the same word (the PTX model gives no
+  // ordering through the address dependency alone); the AND itself can then stay relaxed.
+  static constexpr bool kAcquirePop = true;
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // the 32-bit word holding w's state byte (prefilter and CAS guess)
   const uint32_t* __restrict__ row_ptr;
@@ -177,8 +180,7 @@ struct BfsByteApp {
     start = __ldg(row_ptr + v);
     const uint32_t end = __ldg(row_ptr + v + 1);
     const uint32_t sh = (v & 3u) * 8u;
-    // relaxed: the RMW returns the latest depth in coherence order, and nothing else the
-    // pusher wrote is read (no acquire, so no L1 invalidation per pop)
+    // relaxed RMW: the acquire slot load already ordered it after the pusher's CAS
     const uint32_t d = (atomicAnd(word_of(v), ~(kBInq << sh)) >> sh) & 0x7Fu;
     deg = end - start;
     p = d + 1;
@@ -225,7 +227,7 @@ struct BfsByteApp {
 // atomic), which keeps "residue[v] > eps  =>  v queued or in flight".
 template <bool PART>
 struct PrAppT {
-  static constexpr bool kAcquirePop = false;  // residue taken with atomicExch (RMW)
+  static constexpr bool kAcquirePop = true;  // atomicExch must follow the pusher's crossing add
   using Payload = double;  // delta = alpha * rho / deg(v)
   using Token = double;    // residue before our atomicAdd
   const uint32_t* __restrict__ row_ptr;
@@ -282,7 +284,7 @@ struct PrAppT {
 };
 
 using BfsApp = BfsAppT<false>;
-using BfsDedupeApp = BfsAppT<false, false>;  // u32 state, dedupe mode: relaxed pops
+using BfsDedupeApp = BfsAppT<false, true>;  // u32 state, dedupe mode (acquire pops, see BfsByteApp)
 using BfsPartApp = BfsAppT<true>;
 using PrApp = PrAppT<false>;
 using PrPartApp = PrAppT<true>;

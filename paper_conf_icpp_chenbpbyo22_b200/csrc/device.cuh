@@ -240,11 +240,10 @@ __device__ __forceinline__ void publish_one(const Ring& q, unsigned long long id
 // Try to take the item of index idx: 1 = taken (*item set, slot freed for the
 // next lap), 0 = not published yet, -1 = the item was stolen by a lap-blocked
 // producer (drop the claim).
-// ACQ = false (apps whose per-item state is only touched through RMWs, e.g. the
-// BFS state word and the PageRank residue): relaxed load and CAS -- no L1
-// invalidation (CCTL.IVALL) or MEMBAR per consumed item.  The item id itself is
-// the only payload; everything the consumer then reads about the vertex comes
-// from an atomic RMW, which always observes the latest value in coherence order.
+// ACQ = false: relaxed load and CAS (no CCTL.IVALL / MEMBAR per consumed item).
+// Only valid for an app that reads nothing the pusher wrote before publishing:
+// without the acquire, the PTX model does not order the consumer's later RMWs
+// after the pusher's writes (every app in this library uses ACQ = true).
 template <bool ACQ = true>
 __device__ __forceinline__ int try_consume(const Ring& q, unsigned long long idx, uint32_t* item) {
   unsigned long long* slot = q.slots + (idx & q.mask);
