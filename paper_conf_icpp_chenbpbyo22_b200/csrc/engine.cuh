@@ -80,6 +80,33 @@ constexpr uint32_t kBigNextBits = 20, kBigChunkBits = 20;
   do {                      \
   } while (0)
 #endif
+// Phase profile (tools only: build with -DATOS_PHASE_PROF): thread 0 of each CTA
+// worker accumulates clock64() per phase of the batch loop; the host prints the
+// totals after the launch when ATOS_PHASE is set.
+#ifdef ATOS_PHASE_PROF
+enum { PH_BIG = 0, PH_CLAIM, PH_GATHER, PH_IDLE, PH_BEGIN, PH_SCAN, PH_EXPAND, PH_COMPLETE, PH_NB_LO, PH_NB_HI,
+       PH_EXP_LO, PH_EXP_HI, PH_EDGES_LO, PH_EDGES_HI, PH_N };
+static __device__ unsigned long long g_phase[PH_N];
+#define ATOS_PH_DECL unsigned long long ph_last, ph_acc[PH_N];
+#define ATOS_PH(i)                                                   \
+  do {                                                               \
+    if (threadIdx.x == 0) {                                          \
+      const unsigned long long _n = clock64();                       \
+      ph_acc[i] += _n - ph_last;                                     \
+      ph_last = _n;                                                  \
+    }                                                                \
+  } while (0)
+#define ATOS_PH_FLUSH()                                                  \
+  do {                                                                   \
+    if (threadIdx.x == 0)                                                \
+      for (int _i = 0; _i < PH_N; ++_i) atomicAdd(&g_phase[_i], ph_acc[_i]); \
+  } while (0)
+#else
+#define ATOS_PH_DECL
+#define ATOS_PH(i) do {} while (0)
+#define ATOS_PH_FLUSH() do {} while (0)
+#endif
+
 __host__ __device__ constexpr unsigned long long big_pack(uint32_t gen, uint32_t nchunks, uint32_t next) {
   return ((unsigned long long)(gen & 0xFFFFFFu) << 40) | ((unsigned long long)nchunks << 20) | next;
 }
@@ -325,6 +352,7 @@ struct Worker {
   unsigned backoff;
   unsigned long long idle_since;
   unsigned long long deadline;
+  ATOS_PH_DECL
 
   __device__ __forceinline__ void init(unsigned char* arena, const EngineParams& P) {
     const uint32_t nwarps = blockDim.x >> 5;
@@ -340,6 +368,10 @@ struct Worker {
     idle_since = 0;
     deadline = P.timeout_ns ? globaltimer() + P.timeout_ns : 0;
     if (r == 0) s.ctr[1] = 0;
+#ifdef ATOS_PHASE_PROF
+    ph_last = clock64();
+    for (int i = 0; i < PH_N; ++i) ph_acc[i] = 0;
+#endif
     group_sync<MODE>();
   }
 
@@ -404,6 +436,7 @@ struct Worker {
       }
       first = false;
       group_sync<MODE>();
+      ATOS_PH(PH_CLAIM);
       if (s.ctr[3]) return 0;
       // ------------------------------------------------------ 2. gather
       {
@@ -417,6 +450,7 @@ struct Worker {
       const uint32_t npn = s.ctr[2];
       for (uint32_t i = r; i < npn; i += G) s.pend[i] = s.pend2[i];
       group_sync<MODE>();
+      ATOS_PH(PH_GATHER);
       if (nready) {
         if (r == 0) s.ctr[1] = npn;
         idle_since = 0;
@@ -448,6 +482,7 @@ struct Worker {
         }
       }
       group_sync<MODE>();
+      ATOS_PH(PH_IDLE);
       if (s.ctr[3] == 2) return kGoBig;
       if (s.ctr[3]) return 0;
     }
@@ -502,6 +537,12 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
   app.prepare();
   constexpr bool kAssist = PERSIST && MODE != MODE_THREAD;
   const bool assist = kAssist && P.nbig != 0;
+#ifdef ATOS_PHASE_PROF
+  auto& ph_acc = wk.ph_acc;
+  auto& ph_last = wk.ph_last;
+  unsigned long long ph_exp0 = 0;
+  uint32_t ph_total = 0;
+#endif
 
   while (true) {
     // ---------------------------------------------------------- 0. big-task chunks first
@@ -554,9 +595,11 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
         group_sync<MODE>();
         if (r == 0) finish_big_chunk(P, slot, s.ctr[47]);
         group_sync<MODE>();
+        ATOS_PH(PH_BIG);
         continue;
       }
       group_sync<MODE>();
+      ATOS_PH(PH_BIG);
     }
     const uint32_t nready = wk.acquire(P);
     if (nready == kGoBig) continue;
@@ -575,6 +618,7 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
       s.pay[k] = p;
     }
     group_sync<MODE>();
+    ATOS_PH(PH_BEGIN);
     my_pops += (r == 0) ? nready : 0;
     const uint32_t deferred = s.ctr[5];
 
@@ -613,6 +657,11 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
         }
         __syncthreads();
       }
+      ATOS_PH(PH_SCAN);
+#ifdef ATOS_PHASE_PROF
+      ph_exp0 = ph_last;
+      ph_total = total;
+#endif
       for (uint32_t base = 0; base < total; base += G * kU) {
         const uint32_t wfirst = base + (r & ~31u) * kU;
         if (wfirst >= total) continue;  // warp-uniform; no collective below is skipped by part of a warp
@@ -748,8 +797,20 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
       }
     }
     pusher.flush(q, P.watchdog_ns);
+#ifdef ATOS_PHASE_PROF
+    if (MODE == MODE_CTA) __syncthreads();
+    ATOS_PH(PH_EXPAND);
+    if (MODE == MODE_CTA && threadIdx.x == 0) {
+      const bool lo = ph_total < 8192;
+      ph_acc[lo ? PH_NB_LO : PH_NB_HI] += 1;
+      ph_acc[lo ? PH_EXP_LO : PH_EXP_HI] += ph_last - ph_exp0;
+      ph_acc[lo ? PH_EDGES_LO : PH_EDGES_HI] += ph_total;
+    }
+#endif
     wk.complete(P, nready - deferred);
+    ATOS_PH(PH_COMPLETE);
   }
+  ATOS_PH_FLUSH();
   flush_stats(q, my_pops, my_edges, lane_id() == 0 ? pusher.total : 0);
 }
 

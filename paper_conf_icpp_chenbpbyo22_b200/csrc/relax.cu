@@ -257,6 +257,20 @@ static int launch_relax(const App& app, const Ring& q, const Resolved& r, Part& 
   const int rc = launch_relax_inner(app, q, r, p, st);
   wt.stop(r.stream);
   if (rc == ATOS_OK && st) st->worker_ms += wt.elapsed();
+#ifdef ATOS_PHASE_PROF
+  if (getenv("ATOS_PHASE")) {
+    unsigned long long h[PH_N] = {};
+    cudaStreamSynchronize(r.stream);
+    cudaMemcpyFromSymbol(h, g_phase, sizeof(h));
+    static const char* nm[PH_N] = {"big", "claim", "gather", "idle", "begin", "scan", "expand", "complete",
+                                   "nb_lo", "nb_hi", "exp_lo", "exp_hi", "edges_lo", "edges_hi"};
+    fprintf(stderr, "[phase]");
+    for (int i = 0; i < PH_N; ++i) fprintf(stderr, " %s=%llu", nm[i], h[i]);
+    fprintf(stderr, "\n");
+    unsigned long long z[PH_N] = {};
+    cudaMemcpyToSymbol(g_phase, z, sizeof(z));
+  }
+#endif
   return rc;
 }
 
