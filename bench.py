@@ -296,7 +296,10 @@ def run_atos(args, ws, rank, local):
         if not args.no_cpu:
             line["cpu_baseline"] = cpu_baseline(g, sources, src_info)
         if not args.no_apps:
-            line["apps"] = run_apps(args, dev, peak)
+            line["apps"] = c5_extras(args, g, csr, sources, flush, peak)
+            del flush
+            torch.cuda.empty_cache()
+            line["apps"].update(run_apps(args, dev, peak))
     elif rank == 0:
         line["e2e"] = None
     if rank == 0:
@@ -359,6 +362,57 @@ def cpu_baseline(g, sources, src_info):
     return {"value": edges / dt / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
             "sample": f"one full serial FIFO BFS (oracle_bfs, gcc -O2) from source {sources[0]} on the same C5 graph",
             "seconds": dt}
+
+
+def c5_extras(args, g, csr, sources, flush, peak):
+    """C5 beyond the headline BFS: PageRank on the same S26 graph (one GPU), and the partitioned
+    protocol of section 8(e) with P loopback partitions on this one GPU (the partitions run one after
+    the other, so the time is the SUM of the per-partition work plus the exchange -- a protocol
+    overhead measurement, not a multi-GPU time)."""
+    import paper_conf_icpp_chenbpbyo22_b200 as atos
+    res = {}
+    out = torch.empty(g.n, dtype=torch.float64, device=g.row_ptr.device)
+    atos.pagerank(csr, 0.85, 1e-6, out=out)
+    ms, wms, pops, edges = [], [], [], []
+    for _ in range(2):
+        flush_l2(flush)
+        torch.cuda.synchronize()
+        _, st = atos.pagerank(csr, 0.85, 1e-6, out=out)
+        ms.append(st["kernel_ms"])
+        wms.append(st["worker_ms"])
+        pops.append(st["pops"])
+        edges.append(st["edges"])
+    wm = float(np.mean(wms))
+    alg = PR_BYTES_PER_POP * np.mean(pops) + PR_BYTES_PER_EDGE * np.mean(edges)
+    res["pagerank_c5"] = {"config": f"C5: RMAT scale {args.scale} ef 16 seed 5 (n={g.n}, m={g.m}), alpha 0.85, "
+                                    "eps 1e-6, 1 GPU", "ms_to_converge": float(np.mean(ms)), "worker_ms": wm,
+                          "pops_per_n": float(np.mean(pops)) / g.n,
+                          "edge_relaxations_per_m": float(np.mean(edges)) / g.m,
+                          "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
+                          "atomics_per_s": float(np.mean(edges)) / (wm / 1e3)}
+    del out
+    torch.cuda.empty_cache()
+    dout = torch.empty(g.n, dtype=torch.int32, device=g.row_ptr.device)
+    ref, _ = atos.bfs(csr, sources[0], out=torch.empty_like(dout))
+    ref = ref.clone()
+    lres = {"note": "P loopback partitions on ONE GPU, run serially (sum of per-partition work + exchange); "
+                    "BFS from the first C5 source; result checked equal to the 1-partition depths"}
+    for P in (2, 4, 8):
+        pc = atos.CSR.from_graph(g, num_parts=P)
+        atos.bfs(pc, sources[0], out=dout)
+        ms = []
+        for _ in range(2):
+            flush_l2(flush)
+            torch.cuda.synchronize()
+            _, st = atos.bfs(pc, sources[0], out=dout)
+            ms.append(st["kernel_ms"])
+        lres[f"bfs_P{P}"] = {"ms": float(np.mean(ms)), "rounds": int(st["rounds"]),
+                             "bytes_exchanged": int(st["bytes_exchanged"]), "edges_per_m": st["edges"] / g.m,
+                             "equal_to_single": bool(torch.equal(dout, ref))}
+        pc.close()
+        torch.cuda.empty_cache()
+    res["partitioned_loopback_c5"] = lres
+    return res
 
 
 def bsp_app(call, flush, g, atos_ms, steps=2):

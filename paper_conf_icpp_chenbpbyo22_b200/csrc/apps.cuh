@@ -1,5 +1,7 @@
 // apps.cuh -- relax policies of the two edge-relax applications.
 #pragma once
+#include <cooperative_groups.h>
+
 #include "device.cuh"
 
 namespace atos {
@@ -38,8 +40,14 @@ struct GhostView {
   uint32_t* touched;
   unsigned long long* ntouched;
   __device__ __forceinline__ bool remote_dyn(uint32_t w) const { return ghost != nullptr && (w - vb) >= nl; }
+  // warp-aggregated: one atomicAdd on the list counter per group of lanes touching together
   __device__ __forceinline__ void touch(uint32_t w) const {
-    touched[atomicAdd(ntouched, 1ull)] = w;
+    namespace cg = cooperative_groups;
+    const cg::coalesced_group grp = cg::coalesced_threads();
+    unsigned long long base = 0;
+    if (grp.thread_rank() == 0) base = atomicAdd(ntouched, (unsigned long long)grp.size());
+    base = grp.shfl(base, 0);
+    touched[base + grp.thread_rank()] = w;
   }
 };
 
@@ -156,7 +164,8 @@ struct BfsAppT {
 // re-runs the traversal with the u32 state (high-diameter graphs).
 constexpr uint32_t kBUnreached = 126u, kBMaxDepth = 125u, kBInq = 0x80u;
 
-struct BfsByteApp {
+template <bool PART>
+struct BfsByteAppT {
   // Acquire pops: the slot load must synchronise with the pusher's release so that the
   // popper's AND is ordered after the pusher's CAS on the same word (the PTX model gives no
   // ordering through the address dependency alone); the AND itself can then stay relaxed.
@@ -168,6 +177,10 @@ struct BfsByteApp {
   uint8_t* state;            // n bytes, padded to a multiple of 4
   uint32_t* status;          // queue control block status word
   unsigned long long pol_first, pol_last;
+  GhostView gv;              // PART: ghost = n_global bytes, bits 0-6 the best depth sent or pending for the
+                             // remote vertex (kBUnreached = none), bit 7 = listed in `touched` this round.
+                             // The depth survives the pack (only bit 7 is cleared), so a remote vertex is
+                             // re-sent only when its depth improves -- the ghost filters across rounds.
 
   __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
   __device__ __forceinline__ void prepare() {
@@ -175,6 +188,10 @@ struct BfsByteApp {
     pol_last = policy_evict_last();
   }
   __device__ __forceinline__ uint32_t* word_of(uint32_t v) const { return (uint32_t*)(state + (v & ~3u)); }
+  __device__ __forceinline__ bool remote(uint32_t w) const { return PART && gv.remote_dyn(w); }
+  __device__ __forceinline__ uint32_t* ghost_word(uint32_t w) const {
+    return (uint32_t*)((uint8_t*)gv.ghost + (w & ~3u));
+  }
 
   __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
     start = __ldg(row_ptr + v);
@@ -192,12 +209,37 @@ struct BfsByteApp {
   }
   __device__ __forceinline__ Token pre(const Payload, uint32_t w) const {
     uint32_t word;
-    asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(word) : "l"(word_of(w)), "l"(pol_last) : "memory");
+    const uint32_t* a = remote(w) ? ghost_word(w) : word_of(PART ? w - gv.vb : w);
+    asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(word) : "l"(a), "l"(pol_last) : "memory");
     return word;
   }
   // A stale word only over-states depths (they only decrease), so skipping on it is safe;
   // the CAS decides everything else.
   __device__ __forceinline__ bool post(const Payload nd, uint32_t w, Token word, uint32_t& out) const {
+    if (remote(w)) {
+      // remote relaxation (S10): min-combine into the ghost byte; list w on its first touch this round
+      const uint32_t sh = (w & 3u) * 8u;
+      uint32_t* gp = ghost_word(w);
+      while (true) {
+        const uint32_t b = (word >> sh) & 0xFFu;
+        if ((b & 0x7Fu) <= nd) return false;  // kBUnreached (126) > every encodable nd
+        const uint32_t old = atomicCAS(gp, word, (word & ~(0xFFu << sh)) | ((nd | kBInq) << sh));
+        if (old == word) {
+          if (!(b & kBInq)) gv.touch(w);
+          return false;
+        }
+        word = old;
+      }
+    }
+    return relax_local(nd, PART ? w - gv.vb : w, word, out);
+  }
+  // an inbound (owner-local) relaxation from the exchange
+  __device__ __forceinline__ bool apply(const Payload nd, uint32_t lw, uint32_t& out) const {
+    uint32_t word;
+    asm volatile("ld.global.u32 %0, [%1];" : "=r"(word) : "l"(word_of(lw)) : "memory");
+    return relax_local(nd, lw, word, out);
+  }
+  __device__ __forceinline__ bool relax_local(const Payload nd, uint32_t w, Token word, uint32_t& out) const {
     const uint32_t sh = (w & 3u) * 8u;
     uint32_t* wp = word_of(w);
     while (true) {
@@ -283,6 +325,8 @@ struct PrAppT {
   }
 };
 
+using BfsByteApp = BfsByteAppT<false>;
+using BfsBytePartApp = BfsByteAppT<true>;
 using BfsApp = BfsAppT<false>;
 using BfsDedupeApp = BfsAppT<false, true>;  // u32 state, dedupe mode (acquire pops, see BfsByteApp)
 using BfsPartApp = BfsAppT<true>;

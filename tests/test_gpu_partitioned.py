@@ -41,8 +41,11 @@ def test_bfs_loopback_mesh(P):
     csr = atos.CSR.from_graph(g.to(DEV), num_parts=P)
     r, c = np.divmod(np.arange(R * C), C)
     for (r0, c0) in ((0, 0), (R // 2, C // 2)):
-        d, st = atos.bfs(csr, r0 * C + c0)
-        np.testing.assert_array_equal(as_u32(d), np.abs(r - r0) + np.abs(c - c0))
+        for knobs in (dict(), dict(depth_state=2)):
+            d, st = atos.bfs(csr, r0 * C + c0, **knobs)
+            np.testing.assert_array_equal(as_u32(d), np.abs(r - r0) + np.abs(c - c0))
+            # byte state unless forced to u32 words; the corner source (depth 215) re-runs with u32 words
+            assert bool(st["flags"] & 1) == (not knobs and r0 == 0)
 
 
 def test_bfs_loopback_directed_and_host_output():
