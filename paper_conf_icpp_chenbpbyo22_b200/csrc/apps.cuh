@@ -178,7 +178,8 @@ struct BfsByteAppT {
   uint32_t* status;          // queue control block status word
   unsigned long long pol_first, pol_last;
   GhostView gv;              // PART: ghost = n_global bytes, bits 0-6 the best depth sent or pending for the
-                             // remote vertex (kBUnreached = none), bit 7 = listed in `touched` this round.
+                             // remote vertex (kBUnreached = none), bit 7 = improved this round (the pack
+                             // scans the ghost bytes for it: no list append, no extra atomic in the relax).
                              // The depth survives the pack (only bit 7 is cleared), so a remote vertex is
                              // re-sent only when its depth improves -- the ghost filters across rounds.
 
@@ -209,6 +210,9 @@ struct BfsByteAppT {
   }
   __device__ __forceinline__ Token pre(const Payload, uint32_t w) const {
     uint32_t word;
+#ifdef ATOS_EXP_SKIP_REMOTE
+    if (remote(w)) return 0u;
+#endif
     const uint32_t* a = remote(w) ? ghost_word(w) : word_of(PART ? w - gv.vb : w);
     asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(word) : "l"(a), "l"(pol_last) : "memory");
     return word;
@@ -217,6 +221,9 @@ struct BfsByteAppT {
   // the CAS decides everything else.
   __device__ __forceinline__ bool post(const Payload nd, uint32_t w, Token word, uint32_t& out) const {
     if (remote(w)) {
+#ifdef ATOS_EXP_SKIP_REMOTE
+      return false;
+#endif
       // remote relaxation (S10): min-combine into the ghost byte; list w on its first touch this round
       const uint32_t sh = (w & 3u) * 8u;
       uint32_t* gp = ghost_word(w);
@@ -224,10 +231,7 @@ struct BfsByteAppT {
         const uint32_t b = (word >> sh) & 0xFFu;
         if ((b & 0x7Fu) <= nd) return false;  // kBUnreached (126) > every encodable nd
         const uint32_t old = atomicCAS(gp, word, (word & ~(0xFFu << sh)) | ((nd | kBInq) << sh));
-        if (old == word) {
-          if (!(b & kBInq)) gv.touch(w);
-          return false;
-        }
+        if (old == word) return false;  // bit 7 marks w for the pack's ghost scan (no list append here)
         word = old;
       }
     }
@@ -311,8 +315,8 @@ struct PrAppT {
   }
   __device__ __forceinline__ bool post(const Payload delta, uint32_t w, Token old, uint32_t& out) const {
     if (remote(w)) {
-      // remote mass: sum into the ghost, list it on first touch this round (delta > 0)
-      if (atomicAdd((double*)gv.ghost + w, delta) == 0.0) gv.touch(w);
+      // remote mass: sum into the ghost (red, no return); the pack lists non-zero ghosts
+      red_add_f64((double*)gv.ghost + w, delta);
       return false;
     }
     return crossing(delta, PART ? w - gv.vb : w, old, out);

@@ -541,6 +541,53 @@ __device__ __forceinline__ void block_range(unsigned long long nt, unsigned long
   e = b + per < nt ? b + per : nt;
 }
 
+// Byte-state BFS ghosts: list every vertex whose ghost byte has bit 7 set
+// (improved this round) -- a coalesced scan of n_global bytes, one list append
+// (atomicAdd) per block.
+__global__ void k_ghost_flags_to_list(const uint32_t* __restrict__ ghost_words, int64_t nwords, uint32_t* touched,
+                                      unsigned long long* ntouched) {
+  __shared__ uint32_t tmp[40];
+  __shared__ unsigned long long s_base;
+  for (int64_t w0 = (int64_t)blockIdx.x * blockDim.x; w0 < nwords; w0 += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = w0 + threadIdx.x;
+    const uint32_t word = i < nwords ? ghost_words[i] : 0u;
+    const uint32_t fl = word & 0x80808080u;
+    const uint32_t cnt = __popc(fl);
+    uint32_t tot = 0;
+    const uint32_t ex = block_exclusive_scan(cnt, tmp, &tot);  // uniform trip count: every thread calls it
+    if (tot == 0) continue;
+    if (threadIdx.x == 0) s_base = atomicAdd(ntouched, (unsigned long long)tot);
+    __syncthreads();
+    uint32_t k = 0;
+#pragma unroll
+    for (int b = 0; b < 4; ++b)
+      if (fl & (0x80u << (8 * b))) touched[s_base + ex + k++] = (uint32_t)(4 * i + b);
+    __syncthreads();
+  }
+}
+
+// PageRank ghosts: list every REMOTE vertex (outside [vb, vb+nl)) whose ghost
+// mass is non-zero -- the relax adds remote mass with red.add (no return, so no
+// first-touch test and no list append in the relax loop).
+__global__ void k_ghost_mass_to_list(const double* __restrict__ ghost, int64_t n, int64_t vb, int64_t nl,
+                                     uint32_t* touched, unsigned long long* ntouched) {
+  __shared__ uint32_t tmp[40];
+  __shared__ unsigned long long s_base;
+  const int64_t nr = n - nl;  // remote ids: r < vb -> r, else r + nl
+  for (int64_t r0 = (int64_t)blockIdx.x * blockDim.x; r0 < nr; r0 += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = r0 + threadIdx.x;
+    const int64_t w = r < vb ? r : r + nl;
+    const uint32_t f = (r < nr && ghost[w] != 0.0) ? 1u : 0u;
+    uint32_t tot = 0;
+    const uint32_t ex = block_exclusive_scan(f, tmp, &tot);
+    if (tot == 0) continue;
+    if (threadIdx.x == 0) s_base = atomicAdd(ntouched, (unsigned long long)tot);
+    __syncthreads();
+    if (f) touched[s_base + ex] = (uint32_t)w;
+    __syncthreads();
+  }
+}
+
 // count touched ghosts per destination part
 __global__ void k_pack_count(const uint32_t* touched, const unsigned long long* ntouched, uint32_t chunk,
                              unsigned long long* counts, uint32_t P) {
@@ -549,7 +596,13 @@ __global__ void k_pack_count(const uint32_t* touched, const unsigned long long* 
   __syncthreads();
   unsigned long long b, e;
   block_range(*ntouched, b, e);
-  for (unsigned long long i = b + threadIdx.x; i < e; i += blockDim.x) atomicAdd(s_cnt + touched[i] / chunk, 1u);
+  for (unsigned long long i0 = b; i0 < e; i0 += blockDim.x) {  // uniform trip count: warp-collective below
+    const unsigned long long i = i0 + threadIdx.x;
+    const bool valid = i < e;
+    const uint32_t owner = valid ? touched[i] / chunk : 0xFFFFFFFFu;
+    const unsigned same = __match_any_sync(0xffffffffu, owner);
+    if (valid && (__ffs(same) - 1) == (int)lane_id()) atomicAdd(s_cnt + owner, (unsigned)__popc(same));
+  }
   __syncthreads();
   for (uint32_t d = threadIdx.x; d < P; d += blockDim.x)
     if (s_cnt[d]) atomicAdd(counts + d, (unsigned long long)s_cnt[d]);
@@ -599,16 +652,31 @@ __global__ void k_pack_write(const uint32_t* touched, unsigned long long* ntouch
   __syncthreads();
   unsigned long long b, e;
   block_range(*ntouched, b, e);
-  for (unsigned long long i = b + threadIdx.x; i < e; i += blockDim.x) atomicAdd(s_cnt + touched[i] / chunk, 1u);
+  for (unsigned long long i0 = b; i0 < e; i0 += blockDim.x) {
+    const unsigned long long i = i0 + threadIdx.x;
+    const bool valid = i < e;
+    const uint32_t owner = valid ? touched[i] / chunk : 0xFFFFFFFFu;
+    const unsigned same = __match_any_sync(0xffffffffu, owner);
+    if (valid && (__ffs(same) - 1) == (int)lane_id()) atomicAdd(s_cnt + owner, (unsigned)__popc(same));
+  }
   __syncthreads();
   for (uint32_t d = threadIdx.x; d < P; d += blockDim.x)
     s_cur[d] = s_cnt[d] ? atomicAdd(cursor + d, (unsigned long long)s_cnt[d]) : 0ull;
   __syncthreads();
-  for (unsigned long long i = b + threadIdx.x; i < e; i += blockDim.x) {
-    const uint32_t w = touched[i], owner = w / chunk;
-    const unsigned long long pos = atomicAdd(s_cur + owner, 1ull);
-    out_vid[pos] = w - owner * chunk;
-    out_val[pos] = take(ghost[w]);
+  for (unsigned long long i0 = b; i0 < e; i0 += blockDim.x) {
+    const unsigned long long i = i0 + threadIdx.x;
+    const bool valid = i < e;
+    const uint32_t w = valid ? touched[i] : 0u, owner = valid ? w / chunk : 0xFFFFFFFFu;
+    const unsigned same = __match_any_sync(0xffffffffu, owner);
+    const int leader = __ffs(same) - 1;
+    unsigned long long base = 0;
+    if (valid && leader == (int)lane_id()) base = atomicAdd(s_cur + owner, (unsigned long long)__popc(same));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (valid) {
+      const unsigned long long pos = base + __popc(same & ((1u << lane_id()) - 1u));
+      out_vid[pos] = w - owner * chunk;
+      out_val[pos] = take(ghost[w]);
+    }
   }
 }
 
@@ -653,7 +721,7 @@ __global__ void k_pr_init_edges_part(const uint32_t* __restrict__ row_ptr, const
       const uint32_t w = __ldg(col + e);
       const double add = c / (double)deg;
       if (gv.remote_dyn(w)) {
-        if (atomicAdd((double*)gv.ghost + w, add) == 0.0) gv.touch(w);
+        red_add_f64((double*)gv.ghost + w, add);  // listed by the pack's ghost scan
       } else {
         red_add_f64(res + (w - gv.vb), add);
       }
@@ -680,6 +748,8 @@ namespace {
 
 struct PartRun {
   Part* p;
+  int scan_flags = 0;  // build the touched list from the ghost first: 1 byte bit-7 flags (BFS), 2 non-zero mass (PR)
+  int64_t ghost_words = 0;  // words of ghost bytes to scan (n_global bytes, rounded up)
   uint32_t* state;      // depth (u32) or rank (f64) -- local slice of the output
   GhostView gv;
   unsigned long long* counts;   // device: P counts, then P cursors
@@ -689,6 +759,15 @@ struct PartRun {
 template <class G, class V, class Take>
 int pack_part(PartRun& pr, uint32_t chunk, uint32_t P, Take take, ExchangeIO& io, cudaStream_t s) {
   Part& p = *pr.p;
+  if (pr.scan_flags == 1) {
+    k_ghost_flags_to_list<<<148 * 8, 256, 0, s>>>((const uint32_t*)pr.gv.ghost, pr.ghost_words,
+                                                  p.touched.as<uint32_t>(), pr.ntouched);
+    ++g_launches;
+  } else if (pr.scan_flags == 2) {
+    k_ghost_mass_to_list<<<148 * 8, 256, 0, s>>>((const double*)pr.gv.ghost, pr.ghost_words, (int64_t)pr.gv.vb,
+                                                 (int64_t)pr.gv.nl, p.touched.as<uint32_t>(), pr.ntouched);
+    ++g_launches;
+  }
   ATOS_CUDA(cudaMemsetAsync(pr.counts, 0, sizeof(unsigned long long) * P, s));
   k_pack_count<<<592, 256, P * 4, s>>>(p.touched.as<uint32_t>(), pr.ntouched, chunk, pr.counts, P);
   k_pack_scan<<<1, 32, 0, s>>>(pr.counts, pr.counts + P, P);
@@ -888,6 +967,8 @@ static int bfs_partitioned_bytes(atos_csr* g, int64_t src, uint32_t* depth_out, 
     ATOS_CUDA(cudaMemsetAsync(pk, 0, sizeof(unsigned long long) * (2 * P + 2), s));
     PartRun& pr = runs[i];
     pr.p = &p;
+    pr.scan_flags = 1;
+    pr.ghost_words = (g->n + 3) / 4;
     pr.state = g->comm ? depth_out : depth_out + p.v_begin;
     pr.counts = pk;
     pr.ntouched = pk + 2 * P;
@@ -995,6 +1076,8 @@ int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_out
     pr.counts = pk;
     pr.ntouched = pk + 2 * P;
     pr.gv = GhostView{(uint32_t)p.v_begin, (uint32_t)n, p.ghost_a.p, p.touched.as<uint32_t>(), pr.ntouched};
+    pr.scan_flags = 2;
+    pr.ghost_words = g->n;  // elements (f64)
     Ring q = ring_of(p);
     k_run_begin<<<1, 32, 0, s>>>(q.ctl);
     if (n) {
