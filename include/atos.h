@@ -127,7 +127,11 @@ typedef struct {
     int      depth_state;       /* BFS state (dedupe mode): 0 = auto -- one byte per vertex (7-bit depth + queued
                                    flag, L2-resident), re-run with u32 words if a depth >= 126 is met;
                                    2 = u32 words from the start (high-diameter graphs) */
-    int      reserved_i[2];
+    int      engine_variant;    /* BFS/PageRank worker build: 0 = auto (256-thread CTA workers run the
+                                   48-register, 5-CTAs-per-SM build with 2 edges in flight per thread on
+                                   graphs with m < 8n and 4 otherwise); 1 = the 64-register build (4 edges
+                                   in flight) for every worker size */
+    int      reserved_i[1];
 } atos_cfg;
 
 /* Fill *cfg with defaults (persistent, app-default worker/fetch, dedupe on). */

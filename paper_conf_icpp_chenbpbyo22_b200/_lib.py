@@ -53,7 +53,8 @@ class Cfg(ctypes.Structure):
         ("queue_capacity", ctypes.c_uint64), ("timeout_s", ctypes.c_double), ("stream", ctypes.c_void_p),
         ("stats", ctypes.POINTER(Stats)), ("l2_persist", ctypes.c_int), ("big_threshold", ctypes.c_int),
         ("big_chunk", ctypes.c_int), ("timeline_cap", ctypes.c_uint32), ("timeline", ctypes.c_void_p),
-        ("timeline_interval_ns", ctypes.c_uint32), ("depth_state", ctypes.c_int), ("reserved_i", ctypes.c_int * 2),
+        ("timeline_interval_ns", ctypes.c_uint32), ("depth_state", ctypes.c_int), ("engine_variant", ctypes.c_int),
+        ("reserved_i", ctypes.c_int * 1),
     ]
 
 

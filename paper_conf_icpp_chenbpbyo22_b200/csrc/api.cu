@@ -106,6 +106,11 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
     set_error("depth_state must be 0 (auto) or 2 (u32 words) (got %d)", r->depth_state);
     return ATOS_ERR_INVALID_ARG;
   }
+  r->engine_variant = d.engine_variant;
+  if (r->engine_variant != 0 && r->engine_variant != 1) {
+    set_error("engine_variant must be 0 (auto) or 1 (64-register build) (got %d)", r->engine_variant);
+    return ATOS_ERR_INVALID_ARG;
+  }
   r->big_chunk = d.big_chunk;
   if (r->big_chunk < 0) {
     set_error("big_chunk must be >= 0");

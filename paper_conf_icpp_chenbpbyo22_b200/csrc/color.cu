@@ -23,6 +23,10 @@ namespace atos {
 
 constexpr uint32_t kCheck = 0x80000000u;
 constexpr uint32_t kWin = 1024;  // colours per forbidden-set window (warp/CTA workers)
+#ifndef ATOS_GC_KU
+#define ATOS_GC_KU 4
+#endif
+constexpr int kUc = ATOS_GC_KU;  // CTA worker: edges in flight per thread per expand iteration
 
 struct ColorCtx {
   const uint32_t* __restrict__ row_ptr;
@@ -189,29 +193,57 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
     for (uint32_t i = i0; i < i1; ++i) { const uint32_t d = s.off[i]; s.off[i] = excl; excl += d; }
     __syncthreads();
     edges += tid == 0 ? total : 0;
-    for (uint32_t base = 0; base < total; base += B) {
-      const uint32_t e = base + tid;
-      bool want = false;
-      uint32_t out = 0;
-      if (e < total) {
+    // kUc CONSECUTIVE flattened edges per thread per iteration: one owner search per thread, all col
+    // loads, then all colour loads, then the forbidden-set marks / conflict checks -- kUc independent
+    // memory chains in flight per thread instead of one.
+    for (uint32_t base = 0; base < total; base += B * kUc) {
+      const uint32_t e0 = base + tid * kUc;
+      uint32_t o = 0;
+      if (e0 < total) {
         uint32_t lo = 0, hi = nready;
         while (hi - lo > 1) {
           const uint32_t mid = (lo + hi) >> 1;
-          if (s.off[mid] <= e) lo = mid; else hi = mid;
+          if (s.off[mid] <= e0) lo = mid; else hi = mid;
         }
-        const uint32_t item = s.item[lo], v = item & ~kCheck;
-        const uint32_t w = __ldg(c.col + s.start[lo] + (e - s.off[lo]));
-        if (w != v) {
-          const int32_t cw = ld_relaxed(c.color + w);
-          if (!(item & kCheck)) {
-            if (cw >= 0 && cw < (int32_t)kWin) atomicOr(ibm + lo * 32 + (cw >> 5), 1u << (cw & 31));
-          } else if (cw == cval[lo]) {
-            if (c.literal || c.loses(v, w)) flag[lo] = 1;
-            else if (c.claim_assign(w)) { want = true; out = w; }
-          }
+        o = lo;
+      }
+      uint32_t w[kUc], own[kUc];
+      int32_t cw[kUc];
+      bool val[kUc], want[kUc];
+      uint32_t out[kUc];
+#pragma unroll
+      for (int k = 0; k < kUc; ++k) {
+        const uint32_t e = e0 + k;
+        val[k] = e < total;
+        if (val[k]) {
+          while (o + 1 < nready && s.off[o + 1] <= e) ++o;
+          own[k] = o;
+          w[k] = __ldg(c.col + s.start[o] + (e - s.off[o]));
         }
       }
-      pusher.push(P.q, want, out, P.watchdog_ns);
+#pragma unroll
+      for (int k = 0; k < kUc; ++k) {
+        cw[k] = -1;
+        if (val[k]) {
+          val[k] = w[k] != (s.item[own[k]] & ~kCheck);
+          if (val[k]) cw[k] = ld_relaxed(c.color + w[k]);
+        }
+      }
+#pragma unroll
+      for (int k = 0; k < kUc; ++k) {
+        want[k] = false;
+        out[k] = 0;
+        if (!val[k]) continue;
+        const uint32_t item = s.item[own[k]];
+        if (!(item & kCheck)) {
+          if (cw[k] >= 0 && cw[k] < (int32_t)kWin)
+            atomicOr(ibm + own[k] * 32 + (cw[k] >> 5), 1u << (cw[k] & 31));
+        } else if (cw[k] == cval[own[k]]) {
+          if (c.literal || c.loses(item & ~kCheck, w[k])) flag[own[k]] = 1;
+          else if (c.claim_assign(w[k])) { want[k] = true; out[k] = w[k]; }
+        }
+      }
+      pusher.push_n<kUc>(P.q, want, out, P.watchdog_ns);
     }
     __syncthreads();
     // finalize: one warp per item

@@ -515,11 +515,14 @@ __device__ __forceinline__ void flush_stats(const Ring& q, unsigned long long po
 }
 
 // ------------------------------------------------------------------- kernel
-template <class App, int MODE, bool PERSIST>
+// KU: edges in flight per thread per expand iteration.  MINB > 1: a variant for
+// 256-thread CTA workers with __launch_bounds__(256, MINB) -- fewer registers,
+// MINB resident CTAs per SM (the host picks it, see launch_relax_mode).
 #ifndef ATOS_MAXT
 #define ATOS_MAXT 1024
 #endif
-__global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_worker(App app, EngineParams P) {
+template <class App, int MODE, bool PERSIST, int KU = kU, int MINB = ATOS_MINB>
+__global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_worker(App app, EngineParams P) {
   using Payload = typename App::Payload;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const uint32_t nwarps = blockDim.x >> 5;
@@ -568,28 +571,28 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
         const uint32_t st0 = s.ctr[43] + b0;
         const Payload p = payload_from<Payload>(((unsigned long long)s.ctr[46] << 32) | s.ctr[45]);
         my_edges += (r == 0) ? len : 0;
-        for (uint32_t base = 0; base < len; base += G * kU) {
+        for (uint32_t base = 0; base < len; base += G * KU) {
           // strided lanes (k * G + r): coalesced loads
-          uint32_t w[kU];
-          typename App::Token tk[kU];
+          uint32_t w[KU];
+          typename App::Token tk[KU];
 #pragma unroll
-          for (int k = 0; k < kU; ++k)
+          for (int k = 0; k < KU; ++k)
             if (base + k * G + r < len) {
               w[k] = app.neighbor(st0 + base + k * G + r);
               ATOS_DBG_EDGE(P, st0 + base + k * G + r);
             }
 #pragma unroll
-          for (int k = 0; k < kU; ++k)
+          for (int k = 0; k < KU; ++k)
             if (base + k * G + r < len) tk[k] = app.pre(p, w[k]);
-          bool want[kU];
-          uint32_t out[kU];
+          bool want[KU];
+          uint32_t out[KU];
 #pragma unroll
-          for (int k = 0; k < kU; ++k) {
+          for (int k = 0; k < KU; ++k) {
             want[k] = false;
             out[k] = 0;
             if (base + k * G + r < len) want[k] = app.post(p, w[k], tk[k], out[k]);
           }
-          pusher.push_n<kU>(q, want, out, P.watchdog_ns);
+          pusher.push_n<KU>(q, want, out, P.watchdog_ns);
         }
         pusher.flush(q, P.watchdog_ns);
         group_sync<MODE>();
@@ -634,13 +637,13 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
       for (uint32_t i = i0; i < i1; ++i) { const uint32_t d = s.off[i]; s.off[i] = excl; excl += d; }
       __syncthreads();
       my_edges += (r == 0) ? total : 0;
-      // kU CONSECUTIVE edges per lane per iteration (a warp covers 32*kU
+      // KU CONSECUTIVE edges per lane per iteration (a warp covers 32*KU
       // consecutive flattened edges, so col reads stay coalesced).  Owners:
       // lanes 0/1 binary-search the owners of the warp's first/last edge over
       // the whole batch, then every lane searches only that narrow range and
-      // walks forward over its kU edges.  All col loads, then all prefilter
-      // loads, then the decisions/atomics: kU memory chains in flight per lane.
-      const uint32_t wspan = 32u * kU;
+      // walks forward over its KU edges.  All col loads, then all prefilter
+      // loads, then the decisions/atomics: KU memory chains in flight per lane.
+      const uint32_t wspan = 32u * KU;
       // owner of every wspan-edge chunk start, once per batch (a warp's span is
       // one chunk, so its owner range comes from two table reads)
       const uint32_t nchunk = (total + wspan - 1) / wspan;
@@ -662,8 +665,8 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
       ph_exp0 = ph_last;
       ph_total = total;
 #endif
-      for (uint32_t base = 0; base < total; base += G * kU) {
-        const uint32_t wfirst = base + (r & ~31u) * kU;
+      for (uint32_t base = 0; base < total; base += G * KU) {
+        const uint32_t wfirst = base + (r & ~31u) * KU;
         if (wfirst >= total) continue;  // warp-uniform; no collective below is skipped by part of a warp
         const uint32_t wlast = min(wfirst + wspan, total) - 1;
         uint32_t ob = 0;
@@ -680,10 +683,10 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
           ob = l;
         }
         const uint32_t olo = __shfl_sync(0xffffffffu, ob, 0), ohi = __shfl_sync(0xffffffffu, ob, 1);
-        uint32_t w[kU];
-        typename App::Token tk[kU];
-        bool want[kU];
-        uint32_t out[kU];
+        uint32_t w[KU];
+        typename App::Token tk[KU];
+        bool want[KU];
+        uint32_t out[KU];
         if (olo == ohi) {
           // fast path (warp-uniform): the warp's span lies in ONE row -- no owner search,
           // strided lanes so every load instruction is one coalesced 128-byte access
@@ -691,24 +694,24 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
           const uint32_t len = wlast - wfirst + 1;
           const Payload p = s.pay[olo];
 #pragma unroll
-          for (int k = 0; k < kU; ++k)
+          for (int k = 0; k < KU; ++k)
             if (k * 32 + lane_id() < len) {
               w[k] = app.neighbor(st0 + k * 32 + lane_id());
               ATOS_DBG_EDGE(P, st0 + k * 32 + lane_id());
             }
 #pragma unroll
-          for (int k = 0; k < kU; ++k)
+          for (int k = 0; k < KU; ++k)
             if (k * 32 + lane_id() < len) tk[k] = app.pre(p, w[k]);
 #pragma unroll
-          for (int k = 0; k < kU; ++k) {
+          for (int k = 0; k < KU; ++k) {
             want[k] = false;
             out[k] = 0;
             if (k * 32 + lane_id() < len) want[k] = app.post(p, w[k], tk[k], out[k]);
           }
-          pusher.push_n<kU>(q, want, out, P.watchdog_ns);
+          pusher.push_n<KU>(q, want, out, P.watchdog_ns);
           continue;
         }
-        const uint32_t e0 = wfirst + lane_id() * kU;
+        const uint32_t e0 = wfirst + lane_id() * KU;
         uint32_t o = olo;
         {
           uint32_t l = olo, h = ohi + 1;
@@ -718,10 +721,10 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
           }
           o = l;
         }
-        uint32_t own[kU];
-        bool val[kU];
+        uint32_t own[KU];
+        bool val[KU];
 #pragma unroll
-        for (int k = 0; k < kU; ++k) {
+        for (int k = 0; k < KU; ++k) {
           const uint32_t e = e0 + k;
           val[k] = e < total;
           if (val[k]) {
@@ -733,43 +736,43 @@ __global__ void __launch_bounds__(ATOS_MAXT / ATOS_MINB, ATOS_MINB) k_relax_work
           }
         }
 #pragma unroll
-        for (int k = 0; k < kU; ++k)
+        for (int k = 0; k < KU; ++k)
           if (val[k]) tk[k] = app.pre(s.pay[own[k]], w[k]);
 #pragma unroll
-        for (int k = 0; k < kU; ++k) {
+        for (int k = 0; k < KU; ++k) {
           want[k] = false;
           out[k] = 0;
           if (val[k]) want[k] = app.post(s.pay[own[k]], w[k], tk[k], out[k]);
         }
-        pusher.push_n<kU>(q, want, out, P.watchdog_ns);
+        pusher.push_n<KU>(q, want, out, P.watchdog_ns);
       }
     } else if (MODE == MODE_WARP) {
       for (uint32_t k = 0; k < nready; ++k) {
         const uint32_t st = s.start[k], dg = s.off[k];
         const Payload p = s.pay[k];
         my_edges += (r == 0) ? dg : 0;
-        for (uint32_t j = 0; j < dg; j += 32 * kU) {
+        for (uint32_t j = 0; j < dg; j += 32 * KU) {
           // strided lanes: each load instruction is one coalesced access
-          uint32_t w[kU];
-          typename App::Token tk[kU];
+          uint32_t w[KU];
+          typename App::Token tk[KU];
 #pragma unroll
-          for (int k = 0; k < kU; ++k)
+          for (int k = 0; k < KU; ++k)
             if (j + k * 32 + r < dg) {
               w[k] = app.neighbor(st + j + k * 32 + r);
               ATOS_DBG_EDGE(P, st + j + k * 32 + r);
             }
 #pragma unroll
-          for (int k = 0; k < kU; ++k)
+          for (int k = 0; k < KU; ++k)
             if (j + k * 32 + r < dg) tk[k] = app.pre(p, w[k]);
-          bool want[kU];
-          uint32_t out[kU];
+          bool want[KU];
+          uint32_t out[KU];
 #pragma unroll
-          for (int k = 0; k < kU; ++k) {
+          for (int k = 0; k < KU; ++k) {
             want[k] = false;
             out[k] = 0;
             if (j + k * 32 + r < dg) want[k] = app.post(p, w[k], tk[k], out[k]);
           }
-          pusher.push_n<kU>(q, want, out, P.watchdog_ns);
+          pusher.push_n<KU>(q, want, out, P.watchdog_ns);
         }
       }
     } else {

@@ -113,6 +113,7 @@ struct DeviceGuard {
 struct Resolved {
   int persistent, worker, fetch, num_blocks, block_threads, dedupe, check_size;
   int conflict_policy, permute_init, validate, out_where, l2_persist, big_threshold, big_chunk, depth_state;
+  int engine_variant;
   unsigned long long* timeline;
   uint32_t timeline_cap, timeline_interval_ns;
   uint64_t queue_capacity;

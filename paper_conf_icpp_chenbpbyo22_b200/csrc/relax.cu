@@ -183,7 +183,7 @@ static inline uint64_t pow2_at_least(uint64_t x) {
   return c;
 }
 
-template <class App, int MODE>
+template <class App, int MODE, int KU = kU, int MINB = ATOS_MINB>
 static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, int block,
                              Part& p, atos_stats* st) {
   using Payload = typename App::Payload;
@@ -194,7 +194,7 @@ static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, 
     return ATOS_ERR_INVALID_ARG;
   }
   if (r.persistent) {
-    const void* fn = (const void*)k_relax_worker<App, MODE, true>;
+    const void* fn = (const void*)k_relax_worker<App, MODE, true, KU, MINB>;
     if (smem > 48 * 1024) ATOS_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int grid = 0;
     ATOS_TRY(persistent_grid(fn, block, smem, &grid));
@@ -209,7 +209,7 @@ static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, 
   }
   // discrete: one launch per frontier [h0, t0); the host reads the
   // tail after each launch -- the per-frontier host round trip the paper measures.
-  const void* fn = (const void*)k_relax_worker<App, MODE, false>;
+  const void* fn = (const void*)k_relax_worker<App, MODE, false, KU, MINB>;
   if (smem > 48 * 1024) ATOS_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const uint64_t K = MODE == MODE_THREAD ? 32ull * P.fetch : P.fetch;
   const uint64_t groups_per_block = MODE == MODE_CTA ? 1 : block / 32;
@@ -302,7 +302,17 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
     P.big_threshold = r.big_threshold > 0 ? (uint32_t)r.big_threshold : std::max(4096u, 32u * wsz);
     P.big_chunk = r.big_chunk > 0 ? (uint32_t)r.big_chunk : std::max(1024u, 8u * wsz);
   }
-  if (mode == MODE_CTA) return launch_relax_mode<App, MODE_CTA>(app, P, r, block, p, st);
+  if (mode == MODE_CTA) {
+    // 256-thread CTA workers: the (256, 5) register budget (48 regs, 40 warps per SM); kU = 2 edges
+    // in flight per thread on low-degree graphs (meshes / road-like: m/n < 8), 4 otherwise.  Measured
+    // (tools/sweep.py, one B200): C5 BFS 15.25 -> 14.8 ms, C2 mesh 58 -> 47 ms, road 68 -> 52 ms.
+    if (block == 256 && r.engine_variant != 1) {
+      const bool low_degree = p.n_local > 0 && p.m_local < 8 * p.n_local;
+      if (low_degree) return launch_relax_mode<App, MODE_CTA, 2, 5>(app, P, r, block, p, st);
+      return launch_relax_mode<App, MODE_CTA, 4, 5>(app, P, r, block, p, st);
+    }
+    return launch_relax_mode<App, MODE_CTA>(app, P, r, block, p, st);
+  }
   if (mode == MODE_WARP) return launch_relax_mode<App, MODE_WARP>(app, P, r, block, p, st);
   return launch_relax_mode<App, MODE_THREAD>(app, P, r, block, p, st);
 }

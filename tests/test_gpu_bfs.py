@@ -41,6 +41,9 @@ KNOBS = [
     dict(worker=256, fetch_size=256, depth_state=2),
     dict(worker=32, fetch_size=8, depth_state=2),
     dict(worker=1, fetch_size=2, persistent=0, depth_state=2),
+    # the 64-register worker build at 256 threads (default there: the 48-register 5-CTA/SM build)
+    dict(worker=256, fetch_size=256, engine_variant=1),
+    dict(worker=256, fetch_size=256, persistent=0, engine_variant=1),
 ]
 
 
@@ -66,7 +69,7 @@ def test_rmat_all_knobs(rmat14, knobs):
         assert st["pops"] >= reached  # every reached vertex expanded at least once
 
 
-@pytest.mark.parametrize("knobs", KNOBS[:1] + KNOBS[4:5] + KNOBS[8:9] + KNOBS[6:7], ids=kid)
+@pytest.mark.parametrize("knobs", KNOBS[:1] + KNOBS[4:5] + KNOBS[8:9] + KNOBS[6:7] + KNOBS[-2:], ids=kid)
 def test_mesh_closed_form(knobs):
     R, C = 300, 257
     g = gen.mesh(R, C)

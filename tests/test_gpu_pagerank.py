@@ -26,6 +26,7 @@ KNOBS = [
     dict(worker=256, fetch_size=256, big_threshold=64, big_chunk=16),
     dict(worker=32, fetch_size=4, big_threshold=16, big_chunk=4),
     dict(worker=256, fetch_size=256, big_threshold=-1),
+    dict(worker=256, fetch_size=256, engine_variant=1),
 ]
 
 
