@@ -127,7 +127,7 @@ typedef struct {
     int      depth_state;       /* BFS state (dedupe mode): 0 = auto -- one byte per vertex (7-bit depth + queued
                                    flag, L2-resident), re-run with u32 words if a depth >= 126 is met;
                                    2 = u32 words from the start (high-diameter graphs) */
-    int      engine_variant;    /* BFS/PageRank worker build: 0 = auto (256-thread CTA workers run the
+    int      engine_variant;    /* BFS/PageRank worker build: 0 = auto (persistent 256-thread CTA workers run the
                                    48-register, 5-CTAs-per-SM build with 2 edges in flight per thread on
                                    graphs with m < 8n and 4 otherwise); 1 = the 64-register build (4 edges
                                    in flight) for every worker size */
@@ -152,6 +152,25 @@ ATOS_API void atos_cfg_default(atos_cfg* cfg);
  */
 ATOS_API int atos_csr_create(atos_csr** out, int64_t n, int64_t m, const int64_t* row_ptr,
                     const int32_t* col, int where, int device, int num_parts);
+
+/*
+ * atos_csr_create with layout flags.  atos_csr_create(...) == atos_csr_create_ex(..., 0).
+ *   ATOS_LAYOUT_DEGREE: a single-partition graph is stored in the DEGREE LAYOUT -- vertices relabelled
+ *     once, at creation, by descending degree with the 65536 hottest interleaved one per 128-byte line
+ *     of an f64 state array -- so the hubs' per-vertex state is a compact
+ *     L2-resident prefix.  Invisible to the caller: sources are mapped in, outputs are written in the
+ *     caller's vertex ids, colouring seeds its queue in the caller's id order.  Costs two u32[n] maps
+ *     on the device and one output scatter per call.
+ *   ATOS_LAYOUT_AUTO (0): the degree layout when it pays -- an f64 per-vertex array would not fit half
+ *     of L2 (n * 8 > L2 / 2) and the degrees are skewed (max degree >= 32 * max(1, m / n)); else input.
+ *   ATOS_LAYOUT_INPUT: keep the caller's vertex ids.
+ * Partitioned graphs (num_parts > 1) always keep the input ids.
+ */
+#define ATOS_LAYOUT_AUTO 0
+#define ATOS_LAYOUT_INPUT 1
+#define ATOS_LAYOUT_DEGREE 2
+ATOS_API int atos_csr_create_ex(atos_csr** out, int64_t n, int64_t m, const int64_t* row_ptr,
+                                const int32_t* col, int where, int device, int num_parts, int flags);
 
 /* Release a handle and all its device memory.  NULL is a no-op. */
 ATOS_API void atos_csr_destroy(atos_csr* g);

@@ -25,7 +25,11 @@ def _ptr(t: torch.Tensor) -> ctypes.c_void_p:
 class CSR:
     """Graph handle (atos_csr).  row_ptr: int64[n+1], col: int32[m], host or CUDA tensors."""
 
-    def __init__(self, row_ptr: torch.Tensor, col: torch.Tensor, device: int = 0, num_parts: int = 1):
+    def __init__(self, row_ptr: torch.Tensor, col: torch.Tensor, device: int = 0, num_parts: int = 1,
+                 layout: str = "auto"):
+        """layout (atos_csr_create_ex): "auto" -- the degree layout when it pays (large, skewed graphs),
+        "degree" -- always, "input" -- keep the caller's ids.  The layout is invisible to callers: ids in
+        and out are the caller's."""
         lib = _lib.load()
         row_ptr = row_ptr.contiguous()
         col = col.contiguous()
@@ -38,15 +42,18 @@ class CSR:
         if col.is_cuda != row_ptr.is_cuda:
             raise ValueError("row_ptr and col must live in the same memory space")
         h = ctypes.c_void_p()
-        rc = lib.atos_csr_create(ctypes.byref(h), self.n, self.m, _ptr(row_ptr), _ptr(col), where, device,
-                                 num_parts)
-        _lib.check(rc, "atos_csr_create")
+        flags = {"auto": _lib.LAYOUT_AUTO, "input": _lib.LAYOUT_INPUT, "degree": _lib.LAYOUT_DEGREE}.get(layout)
+        if flags is None:
+            raise ValueError("layout must be 'auto', 'degree' or 'input'")
+        rc = lib.atos_csr_create_ex(ctypes.byref(h), self.n, self.m, _ptr(row_ptr), _ptr(col), where, device,
+                                    num_parts, flags)
+        _lib.check(rc, "atos_csr_create_ex")
         self._h = h
         self.num_parts = num_parts
 
     @classmethod
-    def from_graph(cls, g, device: int = 0, num_parts: int = 1) -> "CSR":
-        return cls(g.row_ptr, g.col, device=device, num_parts=num_parts)
+    def from_graph(cls, g, device: int = 0, num_parts: int = 1, layout: str = "auto") -> "CSR":
+        return cls(g.row_ptr, g.col, device=device, num_parts=num_parts, layout=layout)
 
     @classmethod
     def _wrap(cls, handle, n, m, device, num_parts):

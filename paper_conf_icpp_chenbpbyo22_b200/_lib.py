@@ -28,8 +28,9 @@ EXPORTS = [
     "atos_cfg_default", "atos_csr_create", "atos_csr_destroy", "atos_csr_info", "atos_bfs",
     "atos_pagerank", "atos_color", "atos_comm_unique_id", "atos_comm_create", "atos_comm_destroy",
     "atos_csr_create_part", "atos_partition_range", "atos_last_error", "atos_version",
-    "atos_kernel_launches", "atos_bfs_bsp", "atos_pagerank_bsp", "atos_color_bsp",
+    "atos_kernel_launches", "atos_bfs_bsp", "atos_pagerank_bsp", "atos_color_bsp", "atos_csr_create_ex",
 ]
+LAYOUT_AUTO, LAYOUT_INPUT, LAYOUT_DEGREE = 0, 1, 2
 
 
 class Stats(ctypes.Structure):
@@ -79,6 +80,7 @@ def load(build_if_missing: bool = True):
         sig = {
             "atos_cfg_default": (None, [ctypes.POINTER(Cfg)]),
             "atos_csr_create": (i32, [ctypes.POINTER(P), i64, i64, P, P, i32, i32, i32]),
+            "atos_csr_create_ex": (i32, [ctypes.POINTER(P), i64, i64, P, P, i32, i32, i32, i32]),
             "atos_csr_destroy": (None, [P]),
             "atos_csr_info": (i32, [P, ctypes.POINTER(i64), ctypes.POINTER(i64), ctypes.POINTER(i32)]),
             "atos_bfs": (i32, [P, i64, P, ctypes.POINTER(Cfg)]),

@@ -486,6 +486,22 @@ int create_loopback_parts(atos_csr* g, const int64_t* row_ptr, const int32_t* co
 template <class T>
 int run_with_output(atos_csr* g, T* out, int64_t len, const Resolved& r, DevBuf& staging,
                            const std::function<int(T*)>& body) {
+  if (g->relabeled) {
+    // degree layout: the solver writes internal ids into staging; scatter to the caller's ids
+    ATOS_TRY(staging.ensure((size_t)std::max<int64_t>(len, 1) * sizeof(T)));
+    ATOS_TRY(body(staging.as<T>()));
+    T* dst = out;
+    if (r.out_where != ATOS_MEM_DEVICE) {
+      ATOS_TRY(g->perm_out.ensure((size_t)std::max<int64_t>(len, 1) * sizeof(T)));
+      dst = g->perm_out.as<T>();
+    }
+    ATOS_TRY(layout_scatter<T>(g, staging.as<T>(), dst, r.stream));
+    if (r.out_where != ATOS_MEM_DEVICE) {
+      ATOS_CUDA(cudaMemcpyAsync(out, dst, (size_t)len * sizeof(T), cudaMemcpyDeviceToHost, r.stream));
+      ATOS_CUDA(cudaStreamSynchronize(r.stream));
+    }
+    return ATOS_OK;
+  }
   if (r.out_where == ATOS_MEM_DEVICE) return body(out);
   ATOS_TRY(staging.ensure((size_t)std::max<int64_t>(len, 1) * sizeof(T)));
   ATOS_TRY(body(staging.as<T>()));
@@ -517,8 +533,14 @@ uint64_t atos_kernel_launches(void) { return g_launches.load(); }
 
 int atos_csr_create(atos_csr** out, int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col, int where,
                     int device, int num_parts) {
+  return atos_csr_create_ex(out, n, m, row_ptr, col, where, device, num_parts, ATOS_LAYOUT_AUTO);
+}
+
+int atos_csr_create_ex(atos_csr** out, int64_t n, int64_t m, const int64_t* row_ptr, const int32_t* col, int where,
+                       int device, int num_parts, int flags) {
   if (!out || n < 0 || m < 0 || (n > 0 && !row_ptr) || (m > 0 && !col) || num_parts < 1 ||
-      (where != ATOS_MEM_HOST && where != ATOS_MEM_DEVICE)) {
+      (where != ATOS_MEM_HOST && where != ATOS_MEM_DEVICE) ||
+      (flags != ATOS_LAYOUT_AUTO && flags != ATOS_LAYOUT_INPUT && flags != ATOS_LAYOUT_DEGREE)) {
     set_error("atos_csr_create: invalid argument");
     return ATOS_ERR_INVALID_ARG;
   }
@@ -551,6 +573,16 @@ int atos_csr_create(atos_csr** out, int64_t n, int64_t m, const int64_t* row_ptr
   g->num_parts = num_parts;
   int rc = num_parts == 1 ? create_single(g, row_ptr, col, where) : create_loopback_parts(g, row_ptr, col, where);
   if (rc == ATOS_OK && where == ATOS_MEM_HOST) rc = validate_uploaded_cols(g);
+  if (rc == ATOS_OK && num_parts == 1 && flags != ATOS_LAYOUT_INPUT) {
+    bool want = flags == ATOS_LAYOUT_DEGREE;
+    if (flags == ATOS_LAYOUT_AUTO) {
+      int l2 = 0;
+      cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, device);
+      const int64_t avg = std::max<int64_t>(1, n > 0 ? m / n : 1);
+      want = n * 8 > (int64_t)l2 / 2 && g->max_degree >= 32 * avg;
+    }
+    if (want) rc = layout_by_degree(g);
+  }
   if (rc != ATOS_OK) {
     atos_csr_destroy(g);
     return rc;
@@ -564,6 +596,9 @@ void atos_csr_destroy(atos_csr* g) {
   {
     DeviceGuard dg(g->device);
     for (auto& p : g->parts) destroy_part(p);
+    g->o2n.release();
+    g->n2o.release();
+    g->perm_out.release();
   }
   delete g;
 }
@@ -603,7 +638,11 @@ int atos_bfs(const atos_csr* gc, int64_t src, uint32_t* depth_out, const atos_cf
                                    [&](uint32_t* d) { return bfs_partitioned(g, src, d, r, st); });
   } else {
     rc = run_with_output<uint32_t>(g, depth_out, g->n, r, g->parts[0].vbuf_c,
-                                   [&](uint32_t* d) { return bfs_single(g, g->parts[0], src, d, r, st); });
+                                   [&](uint32_t* d) {
+                                     const int64_t isrc = layout_vertex(g, src);  // degree layout: internal id
+                                     if (isrc < 0) return (int)ATOS_ERR_CUDA;
+                                     return bfs_single(g, g->parts[0], isrc, d, r, st);
+                                   });
     if (st) st->pushes += 1;
   }
   const double ms = tm.stop();
@@ -701,7 +740,11 @@ int atos_bfs_bsp(const atos_csr* gc, int64_t src, uint32_t* depth_out, const ato
   CallTimer tm(r.stream);
   if (g->n == 0) return ATOS_OK;
   int rc = run_with_output<uint32_t>(g, depth_out, g->n, r, g->parts[0].vbuf_c,
-                              [&](uint32_t* d) { return bfs_bsp_single(g, g->parts[0], src, d, r, st); });
+                              [&](uint32_t* d) {
+                                const int64_t isrc = layout_vertex(g, src);
+                                if (isrc < 0) return (int)ATOS_ERR_CUDA;
+                                return bfs_bsp_single(g, g->parts[0], isrc, d, r, st);
+                              });
   const double ms = tm.stop();
   if (rc == ATOS_OK && r.stats) {
     local.kernel_ms = ms;

@@ -412,12 +412,17 @@ __device__ __forceinline__ uint32_t permute_index(uint32_t i, uint32_t n, uint32
 
 // color = -1, every vertex queued as an assign task (Alg.6 line 1
 // "same initialization as Algorithm 5"), in ID order or a seeded permutation.
+// o2n (degree layout, layout.cu): the queue is seeded in the CALLER's vertex-id
+// order (R-GC-6) -- entry i is the internal id of caller vertex i (or of the
+// seeded permutation's i-th vertex).
 __global__ void k_color_init(int32_t* color, uint32_t* inq, Ring q, uint32_t n,
-                             int permute, uint32_t bits, unsigned long long seed, unsigned long long wd) {
+                             int permute, uint32_t bits, unsigned long long seed, unsigned long long wd,
+                             const uint32_t* __restrict__ o2n) {
   const unsigned long long t0 = q.ctl->done.v;  // set to the run's start index by k_color_begin
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     color[i] = -1;
-    const uint32_t v = permute ? permute_index(i, n, bits, seed) : i;
+    uint32_t v = permute ? permute_index(i, n, bits, seed) : i;
+    if (o2n) v = o2n[v];
     publish_one(q, t0 + i, v, wd);
   }
   const uint32_t words = (n + 31) / 32;
@@ -594,7 +599,8 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   uint32_t bits = 1;
   while ((1ull << bits) < n) ++bits;
   if (bits < 2) bits = 2;
-  k_color_init<<<1184, 256, 0, s>>>(color, c.inq, q, n, r.permute_init, bits, seed, r.watchdog_ns);
+  k_color_init<<<1184, 256, 0, s>>>(color, c.inq, q, n, r.permute_init, bits, seed, r.watchdog_ns,
+                                    g->relabeled ? g->o2n.as<uint32_t>() : nullptr);
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   p.ring_clean = false;

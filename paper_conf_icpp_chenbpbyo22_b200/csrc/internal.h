@@ -91,6 +91,8 @@ struct atos_csr {
   int rank = 0, nranks = 1;
   int64_t max_degree = 0;
   bool symmetric_checked = false, symmetric = false;
+  bool relabeled = false;                  // degree layout (layout.cu): internal id = o2n[caller id]
+  atos::DevBuf o2n, n2o, perm_out;         // u32[n] maps; output staging for host outputs
   std::mutex mu;
 };
 
@@ -181,6 +183,12 @@ struct WorkerTimer {
 
 // wait for the stream, honouring cfg.timeout_s (polling) -- returns ATOS_ERR_TIMEOUT on expiry
 int stream_wait(cudaStream_t s, double timeout_s);
+
+// degree layout (layout.cu)
+int layout_by_degree(atos_csr* g);
+template <class T>
+int layout_scatter(const atos_csr* g, const T* in, T* out, cudaStream_t s);
+int64_t layout_vertex(const atos_csr* g, int64_t v);  // caller id -> internal id (-1 on a CUDA error)
 
 // single-partition solvers (relax.cu / color.cu)
 int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth_dev, const Resolved& r,

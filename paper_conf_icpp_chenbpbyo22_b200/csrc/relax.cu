@@ -306,7 +306,7 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
     // 256-thread CTA workers: the (256, 5) register budget (48 regs, 40 warps per SM); kU = 2 edges
     // in flight per thread on low-degree graphs (meshes / road-like: m/n < 8), 4 otherwise.  Measured
     // (tools/sweep.py, one B200): C5 BFS 15.25 -> 14.8 ms, C2 mesh 58 -> 47 ms, road 68 -> 52 ms.
-    if (block == 256 && r.engine_variant != 1) {
+    if (block == 256 && r.persistent && r.engine_variant != 1) {
       const bool low_degree = p.n_local > 0 && p.m_local < 8 * p.n_local;
       if (low_degree) return launch_relax_mode<App, MODE_CTA, 2, 5>(app, P, r, block, p, st);
       return launch_relax_mode<App, MODE_CTA, 4, 5>(app, P, r, block, p, st);

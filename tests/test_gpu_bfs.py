@@ -221,3 +221,30 @@ def test_byte_state_word_neighbours():
     for src in range(12):
         d, _ = atos.bfs(csr, src)
         np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, src))
+
+
+@pytest.mark.parametrize("layout", ["input", "auto", "degree"])
+def test_layout_modes(layout):
+    """The degree layout (default) is invisible: caller ids in, caller ids out, device and host outputs."""
+    g = gen.rmat(13, 16, seed=5)
+    rp, ci = g.numpy()
+    csr = atos.CSR.from_graph(g.to(DEV), layout=layout)
+    for s in (gen.pick_source(g, 9), 0, g.n - 1):
+        want = oracle.bfs(rp, ci, s)
+        d, _ = atos.bfs(csr, s)
+        np.testing.assert_array_equal(as_u32(d), want)
+        out = torch.empty(g.n, dtype=torch.int32)
+        d, _ = atos.bfs(csr, s, out=out)
+        np.testing.assert_array_equal(d.numpy().view(np.uint32), want)
+        d, _ = atos.bfs_bsp(csr, s)
+        np.testing.assert_array_equal(as_u32(d), want)
+
+
+def test_layout_degree_mesh_closed_form():
+    R, C = 300, 257
+    g = gen.mesh(R, C)
+    csr = atos.CSR.from_graph(g.to(DEV), layout="degree")
+    r, c = np.divmod(np.arange(R * C), C)
+    for (r0, c0) in ((0, 0), (R // 2, C // 2)):
+        d, st = atos.bfs(csr, r0 * C + c0)
+        np.testing.assert_array_equal(as_u32(d), np.abs(r - r0) + np.abs(c - c0))

@@ -119,3 +119,15 @@ def test_host_output():
     out = torch.empty(g.n, dtype=torch.int32)
     c, st = atos.color(csr, seed=5, out=out)
     check_color(rp, ci, c, st)
+
+
+@pytest.mark.parametrize("layout", ["input", "auto", "degree"])
+def test_layout_modes_valid(layout):
+    g = gen.rmat(12, 32, seed=8)
+    rp, ci = g.numpy()
+    csr = atos.CSR.from_graph(g.to(DEV), layout=layout)
+    for knobs in (dict(), dict(permute_init=1), dict(worker=32, fetch_size=8)):
+        c, st = atos.color(csr, seed=3, **knobs)
+        check_color(rp, ci, c, st)
+        c, st = atos.color_bsp(csr, seed=3)
+        check_color(rp, ci, c, st)

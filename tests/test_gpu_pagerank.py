@@ -3,6 +3,7 @@ every rank within 1e-4 relative, L1 <= 1e-5 at eps = 1e-6), plus the proven
 one-sided band 0 <= x* - x <= eps x*/(1-a) and mass conservation
 sum x + sum r/(1-a) = n - a #isolated (DESIGN.md R-PR-1/R-PR-6)."""
 import numpy as np
+import torch
 import pytest
 
 import oracle
@@ -107,3 +108,12 @@ def test_bad_args():
         atos.pagerank(csr, 1.0, 1e-6)
     with pytest.raises(RuntimeError, match="INVALID_ARG"):
         atos.pagerank(csr, 0.85, 0.0)
+
+
+def test_layout_input_and_auto_agree(rmat13):
+    rp, ci, ref, _ = rmat13
+    g = gen.Graph(len(rp) - 1, len(ci), torch.from_numpy(rp), torch.from_numpy(ci))
+    for layout in ("input", "auto", "degree"):
+        csr = atos.CSR.from_graph(g.to(DEV), layout=layout)
+        r, st = atos.pagerank(csr, 0.85, 1e-6)
+        check_pr(rp, ci, r, st, 1e-6, ref=ref)
