@@ -269,7 +269,7 @@ def run_atos(args, ws, rank, local):
     achieved = alg_bytes / (w_ms / 1e3) / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": profile_traffic("bfs_worker"), "peak_kind": peak_kind,
-                "kernel": "k_relax_worker<BfsByteApp,CTA,persistent>", "kernel_ms": w_ms,
+                "kernel": "k_relax_worker<BfsByteAppT<0>,CTA,persistent,kU=4,(256,5)>", "kernel_ms": w_ms,
                 "worker_share_of_step": w_ms / ms_per_step}
     gpk = micro_peak("random_gather_per_s")
     if gpk:
@@ -389,7 +389,10 @@ def c5_extras(args, g, csr, sources, flush, peak):
                           "pops_per_n": float(np.mean(pops)) / g.n,
                           "edge_relaxations_per_m": float(np.mean(edges)) / g.m,
                           "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
-                          "atomics_per_s": float(np.mean(edges)) / (wm / 1e3)}
+                          "atomics_per_s": float(np.mean(edges)) / (wm / 1e3),
+                          "traffic": profile_traffic("pr_worker_c5"),
+                          "note": "degree layout (atos_csr_create_ex auto): residue misses L2 less; the f64 "
+                                  "atomics with return are the bound"}
     del out
     torch.cuda.empty_cache()
     dout = torch.empty(g.n, dtype=torch.int32, device=g.row_ptr.device)
@@ -492,7 +495,8 @@ def run_apps(args, dev, peak):
                               "CTA worker 1024 / fetch 128 (library default)",
                     "ms_to_converge": float(np.mean(ms)), "ms_min": float(np.min(ms)), "worker_ms": wm,
                     "colors": int(np.max(cols)), "tasks_per_n": float(np.mean(pops)) / g.n,
-                    "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak}
+                    "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
+                    "traffic": profile_traffic("color_worker")}
     if not args.no_bsp:
         res["color"]["bsp"] = bsp_app(lambda: atos.color_bsp(csr, 1, out=out), flush, g, float(np.mean(ms)))
     del csr, g, out

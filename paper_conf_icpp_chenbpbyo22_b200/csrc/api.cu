@@ -487,15 +487,25 @@ template <class T>
 int run_with_output(atos_csr* g, T* out, int64_t len, const Resolved& r, DevBuf& staging,
                            const std::function<int(T*)>& body) {
   if (g->relabeled) {
-    // degree layout: the solver writes internal ids into staging; scatter to the caller's ids
+    // degree layout: the solver writes internal ids into staging and we scatter to the caller's ids,
+    // unless it wrote the caller's ids itself (r.map_*: the byte-state BFS output pass gathers)
     ATOS_TRY(staging.ensure((size_t)std::max<int64_t>(len, 1) * sizeof(T)));
-    ATOS_TRY(body(staging.as<T>()));
     T* dst = out;
     if (r.out_where != ATOS_MEM_DEVICE) {
       ATOS_TRY(g->perm_out.ensure((size_t)std::max<int64_t>(len, 1) * sizeof(T)));
       dst = g->perm_out.as<T>();
     }
-    ATOS_TRY(layout_scatter<T>(g, staging.as<T>(), dst, r.stream));
+    bool mapped = false;
+    Resolved& rm = const_cast<Resolved&>(r);
+    rm.map_o2n = g->o2n.as<uint32_t>();
+    rm.map_out = dst;
+    rm.map_done = &mapped;
+    const int rc = body(staging.as<T>());
+    rm.map_o2n = nullptr;
+    rm.map_out = nullptr;
+    rm.map_done = nullptr;
+    ATOS_TRY(rc);
+    if (!mapped) ATOS_TRY(layout_scatter<T>(g, staging.as<T>(), dst, r.stream));
     if (r.out_where != ATOS_MEM_DEVICE) {
       ATOS_CUDA(cudaMemcpyAsync(out, dst, (size_t)len * sizeof(T), cudaMemcpyDeviceToHost, r.stream));
       ATOS_CUDA(cudaStreamSynchronize(r.stream));

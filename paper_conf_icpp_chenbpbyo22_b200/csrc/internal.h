@@ -123,6 +123,11 @@ struct Resolved {
   cudaStream_t stream;
   atos_stats* stats;
   unsigned long long watchdog_ns;
+  // degree layout (layout.cu): a solver that can write the CALLER's ids directly (out[j] = f(state[o2n[j]]))
+  // does so into map_out and sets *map_done; otherwise run_with_output scatters its internal-order result.
+  const uint32_t* map_o2n = nullptr;
+  void* map_out = nullptr;
+  bool* map_done = nullptr;
 };
 // defaults: app = 'b' (bfs) / 'p' (pagerank) / 'c' (color)
 int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r);

@@ -66,6 +66,15 @@ __global__ void k_bfs_byte_init(uint8_t* state, Ring q, uint32_t src, unsigned l
   }
 }
 
+// Degree layout: depth_out in the CALLER's ids, gathered (coalesced writes, state bytes read from L2).
+__global__ void k_bfs_byte_output_mapped(const uint8_t* __restrict__ state, const uint32_t* __restrict__ o2n,
+                                         uint32_t* depth, int64_t n) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t D = state[o2n[j]] & 0x7Fu;
+    depth[j] = D == kBUnreached ? 0xFFFFFFFFu : D;
+  }
+}
+
 // depth_out from the byte state (kBUnreached -> 0xFFFFFFFF), 4 vertices per thread.
 __global__ void k_bfs_byte_output(const uint8_t* __restrict__ state, uint32_t* depth, int64_t n) {
   const int64_t nw = (n + 3) / 4;
@@ -351,7 +360,12 @@ static int bfs_single_bytes(Part& p, int64_t src, uint32_t* depth, const Resolve
     *deep = true;
     return ATOS_OK;
   }
-  k_bfs_byte_output<<<148 * 8, 256, 0, s>>>(state, depth, n);
+  if (r.map_o2n && r.map_done) {
+    k_bfs_byte_output_mapped<<<148 * 8, 256, 0, s>>>(state, r.map_o2n, (uint32_t*)r.map_out, n);
+    *r.map_done = true;
+  } else {
+    k_bfs_byte_output<<<148 * 8, 256, 0, s>>>(state, depth, n);
+  }
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   return ATOS_OK;
