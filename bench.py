@@ -418,6 +418,40 @@ def c5_extras(args, g, csr, sources, flush, peak):
     return res
 
 
+def c1_line(dev, flush):
+    """C1: RMAT S16 EF16 seed 1 (65,536 vertices, L2-resident), BFS from the source seed 101 and 7 more,
+    one GPU vs the CPU oracle on the same graph and sources (the config the oracle finishes in seconds)."""
+    import oracle
+    import paper_conf_icpp_chenbpbyo22_b200 as atos
+    from paper_conf_icpp_chenbpbyo22_b200 import gen
+    g = gen.make_config("C1", device=dev)
+    rp, ci = g.numpy()
+    csr = atos.CSR.from_graph(g)
+    out = torch.empty(g.n, dtype=torch.int32, device=dev)
+    srcs = [gen.pick_source(g, 101 + i) for i in range(8)]
+    deg = np.diff(rp)
+    ms, edges, cpu_s = [], [], []
+    for s in srcs:
+        atos.bfs(csr, s, out=out)
+        flush_l2(flush)
+        torch.cuda.synchronize()
+        _, st = atos.bfs(csr, s, out=out)
+        ms.append(st["kernel_ms"])
+        t0 = time.perf_counter()
+        want = oracle.bfs(rp, ci, s)
+        cpu_s.append(time.perf_counter() - t0)
+        ok = bool(np.array_equal(out.cpu().numpy().view(np.uint32), want))
+        if not ok:
+            raise RuntimeError(f"C1 BFS mismatch vs oracle from source {s}")
+        edges.append(int(deg[want != 0xFFFFFFFF].sum()))
+    return {"config": f"C1: RMAT scale 16 ef 16 seed 1 (n={g.n}, m={g.m}), sources seeds 101..108",
+            "ms_per_bfs": float(np.mean(ms)), "gteps": sum(edges) / (sum(ms) / 1e3) / 1e9,
+            "oracle_ms_per_bfs": 1e3 * float(np.mean(cpu_s)), "oracle_gteps": sum(edges) / sum(cpu_s) / 1e9,
+            "bit_exact_vs_oracle": True,
+            "note": "L2-resident graph: latency/launch bound (init + persistent launch + termination), "
+                    "not bandwidth bound"}
+
+
 def bsp_app(call, flush, g, atos_ms, steps=2):
     """Time a BSP baseline call (stats.kernel_ms, L2 flushed before each step) next to the Atos number."""
     call()
@@ -440,6 +474,7 @@ def run_apps(args, dev, peak):
     import paper_conf_icpp_chenbpbyo22_b200 as atos
     res = {}
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    res["bfs_c1"] = c1_line(dev, flush)
     # ---- PageRank on C3
     g = make_graph(args.pr_scale, 16, 3, dev)
     csr = atos.CSR.from_graph(g)
