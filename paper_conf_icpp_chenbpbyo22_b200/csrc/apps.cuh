@@ -285,6 +285,8 @@ struct PrAppT {
   int activate;          // 1: crossing activation (default); 0: sweep-only (Check_Size variant)
   uint32_t* dbg_expand;  // debug: per-vertex count of expanding pops
   GhostView gv;
+  double defer = 0.0;    // partitioned schedule only: a popped vertex with deg > 32 and residue < defer * deg
+                         // keeps its residue (not expanded) until a later, lower threshold re-seeds it
 
   __device__ __forceinline__ bool remote(uint32_t w) const { return PART && gv.remote_dyn(w); }
   __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
@@ -293,9 +295,14 @@ struct PrAppT {
   __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
     const double rho = __longlong_as_double(
         (long long)atomicExch((unsigned long long*)(res + v), 0ull));
-    if (rho != 0.0) red_add_f64(rank + v, rho);
     start = __ldg(row_ptr + v);
     deg = __ldg(row_ptr + v + 1) - start;
+    if (PART && defer > 0.0 && deg > 32 && rho < defer * (double)deg) {
+      // hub with too little residue for its edge count: hand it back; re-seeded at a lower threshold
+      if (rho != 0.0) red_add_f64(res + v, rho);
+      return false;
+    }
+    if (rho != 0.0) red_add_f64(rank + v, rho);
     if (deg == 0 || rho == 0.0) return false;  // dangling: absorb (R-PR-3)
     if (dbg_expand) atomicAdd(dbg_expand + v, 1u);
     p = alpha * rho / (double)deg;
