@@ -506,7 +506,23 @@ def run_apps(args, dev, peak):
     if not args.no_bsp:
         res["pagerank"]["bsp"] = bsp_app(lambda: atos.pagerank_bsp(csr, 0.85, 1e-6, out=out), flush, g,
                                          float(np.mean(ms)))
-    del csr, g, out
+    # the partitioned round protocol (section 8(e)) on C3 with P loopback partitions on this GPU
+    ref = out.clone()
+    pl = {"note": "P loopback partitions on ONE GPU, run serially (sum of per-partition work + exchange); "
+                  "L1 of rank/n vs the single-partition result"}
+    for P in (2, 4, 8):
+        pc = atos.CSR.from_graph(g, num_parts=P)
+        po = torch.empty_like(out)
+        atos.pagerank(pc, 0.85, 1e-6, out=po)
+        flush_l2(flush)
+        torch.cuda.synchronize()
+        _, st = atos.pagerank(pc, 0.85, 1e-6, out=po)
+        pl[f"P{P}"] = {"ms": st["kernel_ms"], "rounds": int(st["rounds"]), "bytes_exchanged": int(st["bytes_exchanged"]),
+                       "edge_relaxations_per_m": st["edges"] / g.m, "l1_vs_single": float((po - ref).abs().sum().item())}
+        pc.close()
+        del po
+    res["pagerank"]["partitioned_loopback"] = pl
+    del csr, g, out, ref
     torch.cuda.empty_cache()
     # ---- colouring on C4
     g = make_graph(args.gc_scale, 64, 4, dev)
