@@ -124,7 +124,11 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
   }
   r->stream = (cudaStream_t)d.stream;
   r->stats = d.stats;
-  r->watchdog_ns = (unsigned long long)((r->timeout_s > 0 ? r->timeout_s : 10.0) * 1e9);
+  // no-progress watchdog: cfg.timeout_s, else 10 s (ATOS_WATCHDOG_S overrides the default -- tools, e.g.
+  // kernels slowed 100x under compute-sanitizer)
+  const char* wd_env = getenv("ATOS_WATCHDOG_S");
+  const double wd_default = wd_env && atof(wd_env) > 0 ? atof(wd_env) : 10.0;
+  r->watchdog_ns = (unsigned long long)((r->timeout_s > 0 ? r->timeout_s : wd_default) * 1e9);
   return ATOS_OK;
 }
 

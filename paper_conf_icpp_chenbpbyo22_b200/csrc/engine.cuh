@@ -485,6 +485,9 @@ struct Worker {
       ATOS_PH(PH_IDLE);
       if (s.ctr[3] == 2) return kGoBig;
       if (s.ctr[3]) return 0;
+      // every member has read s.ctr[3] before the group leader resets it for the next claim
+      // (compute-sanitizer racecheck: WAR on s.ctr[3] across the loop back-edge)
+      group_sync<MODE>();
     }
   }
 
