@@ -179,6 +179,7 @@ def run_reference(args, ws, rank):
     g = make_graph(args.scale, 16, 5, "cuda")
     rp, ci = g.numpy()
     sources = [gen.pick_source(g, 105 + i) for i in range(8)]
+    n, m = g.n, g.m
     del g
     torch.cuda.empty_cache()
     times, edges = [], []
@@ -197,8 +198,10 @@ def run_reference(args, ws, rank):
         "impl": "reference", "metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": ws,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": total / len(times) * 1e3,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-        "config": {"workload": f"C5 BFS RMAT scale {args.scale} ef 16 seed 5, 8 seeded sources",
-                   "global_batch": 1, "parallelism": "serial-oracle"},
+        "config": {"workload": f"C5: BFS on RMAT scale {args.scale} ef 16 seed 5 (n={n}, m={m}), "
+                               f"8 seeded sources, 1D vertex partition over {ws} GPU(s)",
+                   "global_batch": 1, "parallelism": f"vertex-partition{ws}",
+                   "implementation": "serial CPU oracle (oracle/atos_oracle.c, gcc -O2), 1 host core"},
         "cpu_baseline": {"value": value, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                          "sample": f"full serial FIFO BFS (oracle_bfs) from each seeded source, {args.steps} steps"},
         "e2e": {"value": value, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
