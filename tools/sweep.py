@@ -34,6 +34,7 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--grid", default=None)
     ap.add_argument("--extra", default="", help="k=v,k=v knobs added to every configuration")
+    ap.add_argument("--layout", default="auto", help="CSR layout: auto | degree | input")
     a = ap.parse_args()
     extra = {k: int(v) for k, v in (kv.split("=") for kv in a.extra.split(",") if kv)}
     if a.app in ("bfs-mesh", "bfs-road"):
@@ -48,7 +49,7 @@ def main():
     else:
         g = gen.rmat(a.scale or 20, 64, 4, device="cuda")
         src = None
-    csr = atos.CSR.from_graph(g)
+    csr = atos.CSR.from_graph(g, layout=a.layout)
     n, m = g.n, g.m
     del g
     torch.cuda.empty_cache()
