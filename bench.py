@@ -556,7 +556,14 @@ def run_apps(args, dev, peak):
                     "ms_to_converge": float(np.mean(ms)), "ms_min": float(np.min(ms)), "worker_ms": wm,
                     "colors": int(np.max(cols)), "tasks_per_n": float(np.mean(pops)) / g.n,
                     "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
-                    "traffic": profile_traffic("color_worker")}
+                    "traffic": profile_traffic("color_worker"), "edge_visits_per_m": float(np.mean(edges)) / g.m}
+    gpk = micro_peak("random_gather_per_s")
+    if gpk:
+        # every edge visit (assign or check) gathers one neighbour colour: the random-gather ceiling
+        ach = float(np.mean(edges)) / (wm / 1e3)
+        res["color"]["pattern_roofline"] = {"bound": "l1tex random-gather wavefronts (1 colour load per edge visit)",
+                                            "achieved": ach, "peak": gpk, "unit": "gathers/s", "frac": ach / gpk,
+                                            "peak_source": "profiles/r01_micro_peaks.json"}
     if not args.no_bsp:
         res["color"]["bsp"] = bsp_app(lambda: atos.color_bsp(csr, 1, out=out), flush, g, float(np.mean(ms)))
     del csr, g, out
