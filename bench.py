@@ -72,32 +72,56 @@ def profile_traffic(kernel_key: str):
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """nvidia-smi clocks + throttle reasons sampled every 20 ms during the timed region.
+
+    A reader thread collects the rows; __enter__ returns only after nvidia-smi produced its first row (its
+    start-up takes longer than a short timed region), and only rows read between __enter__ and __exit__
+    are kept (plus the first one after, which covers the region's tail)."""
     FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
               "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
     def __init__(self, index: int):
         self.index = index
         self.proc = None
+        self.rows = []
+        self.t_on = self.t_off = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            now = time.monotonic()
+            if self.t_on is not None and (self.t_off is None or not self._tail_taken):
+                if self.t_off is not None:
+                    self._tail_taken = True
+                self.rows.append(line)
+            self._first.set()
 
     def __enter__(self):
+        import threading
+        self._first = threading.Event()
+        self._tail_taken = False
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", "20"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+            self._first.wait(timeout=5.0)
         except Exception:
             self.proc = None
+        self.t_on = time.monotonic()
         return self
 
     def __exit__(self, *a):
-        self.out = ""
+        self.t_off = time.monotonic()
         if self.proc is not None:
-            time.sleep(0.25)
+            time.sleep(0.05)
             self.proc.terminate()
             try:
-                self.out, _ = self.proc.communicate(timeout=5)
+                self.proc.wait(timeout=5)
+                self.thread.join(timeout=2)
             except Exception:
                 self.proc.kill()
+        self.out = "".join(self.rows)
 
     def summary(self):
         rows = [r.split(",") for r in (self.out or "").strip().splitlines() if r.count(",") >= 5]
@@ -528,6 +552,15 @@ def run_apps(args, dev, peak):
         _, st = atos.pagerank(pc, 0.85, 1e-6, out=po)
         pl[f"P{P}"] = {"ms": st["kernel_ms"], "rounds": int(st["rounds"]), "bytes_exchanged": int(st["bytes_exchanged"]),
                        "edge_relaxations_per_m": st["edges"] / g.m, "l1_vs_single": float((po - ref).abs().sum().item())}
+        # NEXT-4 barrier-free protocol on the same partitions: one persistent kernel, remote mass and
+        # activations straight into the owner's slice and queue (all partitions run concurrently)
+        atos.pagerank(pc, 0.85, 1e-6, out=po, barrier_free=1)
+        flush_l2(flush)
+        torch.cuda.synchronize()
+        _, st = atos.pagerank(pc, 0.85, 1e-6, out=po, barrier_free=1)
+        pl[f"P{P}_barrier_free"] = {"ms": st["kernel_ms"], "worker_ms": st["worker_ms"],
+                                    "edge_relaxations_per_m": st["edges"] / g.m, "pops_per_n": st["pops"] / g.n,
+                                    "l1_vs_single": float((po - ref).abs().sum().item())}
         pc.close()
         del po
     res["pagerank"]["partitioned_loopback"] = pl

@@ -55,7 +55,7 @@ class Cfg(ctypes.Structure):
         ("stats", ctypes.POINTER(Stats)), ("l2_persist", ctypes.c_int), ("big_threshold", ctypes.c_int),
         ("big_chunk", ctypes.c_int), ("timeline_cap", ctypes.c_uint32), ("timeline", ctypes.c_void_p),
         ("timeline_interval_ns", ctypes.c_uint32), ("depth_state", ctypes.c_int), ("engine_variant", ctypes.c_int),
-        ("reserved_i", ctypes.c_int * 1),
+        ("barrier_free", ctypes.c_int),
     ]
 
 

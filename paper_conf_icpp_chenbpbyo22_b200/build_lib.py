@@ -11,7 +11,7 @@ CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(HERE, "libatos.so")
-SOURCES = ["api.cu", "relax.cu", "color.cu", "dist.cu", "bsp.cu", "layout.cu"]
+SOURCES = ["api.cu", "relax.cu", "color.cu", "dist.cu", "bsp.cu", "layout.cu", "nobarrier.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "-I", INCLUDE, "-I", CSRC,

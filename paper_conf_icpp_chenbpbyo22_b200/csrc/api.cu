@@ -111,6 +111,11 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
     set_error("engine_variant must be 0 (auto) or 1 (64-register build) (got %d)", r->engine_variant);
     return ATOS_ERR_INVALID_ARG;
   }
+  r->barrier_free = d.barrier_free;
+  if (r->barrier_free != 0 && r->barrier_free != 1) {
+    set_error("barrier_free must be 0 or 1 (got %d)", r->barrier_free);
+    return ATOS_ERR_INVALID_ARG;
+  }
   r->big_chunk = d.big_chunk;
   if (r->big_chunk < 0) {
     set_error("big_chunk must be >= 0");
@@ -686,7 +691,14 @@ int atos_pagerank(const atos_csr* gc, double alpha, double eps, double* rank_out
   CallTimer tm(r.stream);
   int rc;
   if (g->n == 0) return ATOS_OK;
-  if (g->comm || g->num_parts > 1) {
+  if (r.barrier_free) {
+    if (g->comm || g->num_parts < 2) {
+      set_error("atos_pagerank: barrier_free needs a loopback-partitioned graph (num_parts > 1, one process)");
+      return ATOS_ERR_UNSUPPORTED;
+    }
+    rc = run_with_output<double>(g, rank_out, g->n, r, g->parts[0].vbuf_c,
+                                 [&](double* d) { return pagerank_nobarrier(g, alpha, eps, d, r, st); });
+  } else if (g->comm || g->num_parts > 1) {
     const int64_t len = g->comm ? g->parts[0].n_local : g->n;
     rc = run_with_output<double>(g, rank_out, len, r, g->parts[0].vbuf_c,
                                  [&](double* d) { return pagerank_partitioned(g, alpha, eps, d, r, st); });

@@ -53,6 +53,7 @@ struct Part {
   DevBuf ring, ctl, big, bitmap, shadow, vbuf_a, vbuf_b, vbuf_c, scratch;
   DevBuf ghost_a, ghost_b, touched, outbox, inbox, out_val, in_val, pack;
   DevBuf bsp_fa, bsp_fb, bsp_off, bsp_tmp, bsp_ctr;  // BSP baselines (bsp.cu)
+  DevBuf nb_ring, nb_ctl, nb_peers;                   // barrier-free partitioned PageRank (nobarrier.cu)
   uint64_t ring_cap = 0;
   void* host_pinned = nullptr;      // 4 KB pinned scratch for control-block reads
   bool ring_clean = false;          // every ring slot is EMPTY
@@ -116,6 +117,7 @@ struct Resolved {
   int persistent, worker, fetch, num_blocks, block_threads, dedupe, check_size;
   int conflict_policy, permute_init, validate, out_where, l2_persist, big_threshold, big_chunk, depth_state;
   int engine_variant;
+  int barrier_free;
   unsigned long long* timeline;
   uint32_t timeline_cap, timeline_interval_ns;
   uint64_t queue_capacity;
@@ -216,6 +218,9 @@ int color_count(Part& p, const int32_t* color, int64_t* used, cudaStream_t s);
 int bfs_partitioned(atos_csr* g, int64_t src, uint32_t* depth_dev, const Resolved& r, atos_stats* st);
 int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_dev, const Resolved& r,
                          atos_stats* st);
+// barrier-free partitioned PageRank, loopback partitions (nobarrier.cu, NEXT-4)
+int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_dev, const Resolved& r,
+                       atos_stats* st);
 
 // read the control block after a run: status -> error code, stats
 int finish_queue(Part& p, cudaStream_t s, atos_stats* st, const char* what);

@@ -1,0 +1,383 @@
+// nobarrier.cu -- NEXT-4: barrier-free partitioned PageRank.
+//
+// The exchange-round path (relax.cu pagerank_partitioned) runs every partition to local
+// quiescence, then exchanges ghost mass and starts the next round.  Here the barrier goes away, which is
+// the paper's relaxed-barrier thesis applied across partitions: one persistent kernel in
+// which every partition's workers push mass for a REMOTE vertex straight into the owner's residue slice
+// (atomicAdd on the owner's memory -- peer memory over NVLink in a multi-GPU build, the same device in
+// this loopback build) and, on a threshold crossing (Alg.4, R-PR-7), into the owner's queue.
+// Termination is global quiescence: sum(done) == sum(tail) over all partitions, read as every done
+// counter and then every tail counter (monotone counters; an item's pushes are reserved before its done
+// increment, so equal sums imply a moment with nothing queued or in flight anywhere).
+//
+// Worker: a CTA claims up to 256 items of ITS partition's ring (one CAS on head, never past tail), each
+// thread begins one item (atomicExch residue -> rank, delta = alpha*rho/deg, Alg.4), and each
+// warp expands its 32 items' rows load-balanced.  Pushes are warp-aggregated per destination partition
+// (match_any + one atomicAdd on that ring's tail).  Slots carry a lap tag so a consumer never mistakes
+// the previous lap's value for its own item.
+#include "internal.h"
+
+namespace atos {
+
+namespace {
+
+constexpr uint32_t kNbMaxParts = 8;
+constexpr int kNbBlock = 256;
+
+struct NbCtl {  // one per partition; each counter on its own 128-byte line
+  unsigned long long head, pad0[15];
+  unsigned long long tail, pad1[15];
+  unsigned long long done, pad2[15];
+};
+
+struct NbPeer {  // what a partition exposes to its peers (peer-mapped in a multi-GPU build)
+  const uint32_t* row_ptr;  // n_local + 1, local offsets
+  const uint32_t* col;      // GLOBAL ids
+  double* rank;             // n_local (caller's output slice)
+  double* res;              // n_local
+  unsigned long long* ring; // cap slots: 0 = free, else tag(idx) << 32 | local id
+  NbCtl* ctl;
+  unsigned long long mask;  // cap - 1
+  uint32_t n_local, pad;
+};
+
+struct NbGlob {
+  unsigned long long abort;  // set by a watchdog
+  unsigned long long edges;  // neighbour-list entries visited
+};
+
+struct NbParams {
+  const NbPeer* peers;  // device array [P]
+  NbGlob* glob;
+  uint32_t P, B;        // partitions, block size ceil(n / P) (atos_partition_range)
+  double alpha, eps;
+  unsigned long long watchdog_ns;
+};
+
+__device__ __forceinline__ unsigned long long nb_tag(unsigned long long idx, uint32_t item) {
+  // lap tag never 0 (bit 31 set), distinct for idx and idx - cap while cap < 2^31
+  const unsigned long long t = (idx & 0x7FFFFFFFull) | 0x80000000ull;
+  return (t << 32) | item;
+}
+
+__device__ __forceinline__ bool nb_aborted(const NbGlob* g) {
+  return ld_relaxed(&g->abort) != 0ull;
+}
+
+// Warp-aggregated push of `lw` into partition `o`'s ring for the lanes with act set.
+__device__ __forceinline__ void nb_push(const NbParams& prm, bool act, uint32_t o, uint32_t lw) {
+  const unsigned am = __ballot_sync(0xffffffffu, act);
+  if (!am || !act) return;
+  const unsigned grp = __match_any_sync(am, o);
+  const uint32_t lane = lane_id();
+  const int leader = __ffs(grp) - 1;
+  const uint32_t rank = __popc(grp & ((1u << lane) - 1u));
+  const NbPeer* pe = prm.peers + o;
+  NbCtl* c = pe->ctl;
+  unsigned long long base = 0;
+  if ((int)lane == leader) base = atomicAdd(&c->tail, (unsigned long long)__popc(grp));
+  base = __shfl_sync(grp, base, leader);
+  const unsigned long long idx = base + rank;
+  unsigned long long* slot = pe->ring + (idx & pe->mask);
+  // the previous lap's consumer may not have released the slot yet
+  while (ld_relaxed(slot) != 0ull) {
+    if (nb_aborted(prm.glob)) return;
+    __nanosleep(32);
+  }
+  st_release(slot, nb_tag(idx, lw));
+}
+
+}  // namespace
+
+// Rank / residue init of every partition (Alg.3, R-PR-init): rank = 1 - alpha, residue = 0.
+__global__ void k_nb_init_vertices(NbParams prm, double one_minus_alpha) {
+  for (uint32_t p = 0; p < prm.P; ++p) {
+    const NbPeer pe = prm.peers[p];
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < pe.n_local;
+         v += (int64_t)gridDim.x * blockDim.x) {
+      pe.rank[v] = one_minus_alpha;
+      pe.res[v] = 0.0;
+    }
+  }
+}
+
+// residue[w] += alpha*(1-alpha)/deg(v) for every edge v -> w, written into the owner's slice (warp per row).
+__global__ void k_nb_init_edges(NbParams prm, uint32_t p, double c) {
+  const NbPeer pe = prm.peers[p];
+  const uint32_t lane = lane_id();
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t v = blockIdx.x * (int64_t)(blockDim.x >> 5) + warp_id(); v < pe.n_local; v += warps) {
+    const uint32_t s = __ldg(pe.row_ptr + v), deg = __ldg(pe.row_ptr + v + 1) - s;
+    if (!deg) continue;
+    const double add = c / (double)deg;
+    for (uint32_t e = lane; e < deg; e += 32) {
+      const uint32_t w = __ldg(pe.col + s + e);
+      const uint32_t o = w / prm.B;
+      red_add_f64(prm.peers[o].res + (w - o * prm.B), add);
+    }
+  }
+}
+
+// Initial frontier of partition p: every local vertex with residue > eps (R-PR-7).
+__global__ void k_nb_seed(NbParams prm, uint32_t p) {
+  const uint32_t n = prm.peers[p].n_local;
+  const double* res = prm.peers[p].res;
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t base = blockIdx.x * blockDim.x; base < n; base += stride) {
+    const uint32_t v = base + threadIdx.x;
+    nb_push(prm, v < n && res[v] > prm.eps, p, v);
+  }
+}
+
+// The persistent barrier-free worker kernel (one cooperative launch; CTA b serves partition b % P).
+// A CTA claims up to kNbBlock items of its partition's ring with ONE CAS (fewer contenders on head than
+// a claim per warp); warp w takes items [32w, 32w+32) of the batch and expands them load-balanced: a warp
+// scan of the 32 degrees, then every lane takes edge e of the batch's concatenated rows and finds its item
+// by a 5-step search over the 32 row offsets (the warp-level form of the CTA worker's LBS).
+__global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
+  __shared__ unsigned long long s_h;
+  __shared__ uint32_t s_k;
+  __shared__ int s_quit;
+  __shared__ uint32_t s_off[kNbBlock / 32][32], s_start[kNbBlock / 32][32];
+  __shared__ double s_delta[kNbBlock / 32][32];
+  const uint32_t me = blockIdx.x % prm.P;
+  const NbPeer self = prm.peers[me];
+  const uint32_t lane = lane_id(), wid = warp_id();
+  unsigned long long edges = 0, t_idle = 0, last_done = 0;
+  while (true) {
+    if (threadIdx.x == 0) {
+      uint32_t k = 0;
+      unsigned long long h = 0, hh = ld_relaxed(&self.ctl->head);
+      while (true) {
+        const unsigned long long t = ld_relaxed(&self.ctl->tail);
+        if (hh >= t) break;
+        const uint32_t want = (uint32_t)min((unsigned long long)kNbBlock, t - hh);
+        const unsigned long long got = atomicCAS(&self.ctl->head, hh, hh + want);
+        if (got == hh) {
+          h = hh;
+          k = want;
+          break;
+        }
+        hh = got;
+      }
+      int quit = 0;
+      if (k == 0) {
+        if (nb_aborted(prm.glob)) {
+          quit = 1;
+        } else {
+          unsigned long long D = 0, T = 0;
+          for (uint32_t p = 0; p < prm.P; ++p) D += atom_read(&prm.peers[p].ctl->done);
+          for (uint32_t p = 0; p < prm.P; ++p) T += atom_read(&prm.peers[p].ctl->tail);
+          if (D == T) {
+            quit = 1;
+          } else {
+            // watchdog: no partition completed an item for watchdog_ns
+            const unsigned long long now = globaltimer();
+            if (t_idle == 0 || D != last_done) {
+              t_idle = now;
+              last_done = D;
+            } else if (now - t_idle > prm.watchdog_ns) {
+              atomicExch(&prm.glob->abort, 1ull);
+              quit = 1;
+            }
+            __nanosleep(256);
+          }
+        }
+      } else {
+        t_idle = 0;
+      }
+      s_h = h;
+      s_k = k;
+      s_quit = quit;
+    }
+    __syncthreads();
+    const unsigned long long h = s_h;
+    const uint32_t k = s_k;
+    const int quit = s_quit;
+    __syncthreads();
+    if (quit) break;
+    if (k == 0) continue;
+    // consume one claimed slot per thread
+    uint32_t start = 0, deg = 0;
+    double delta = 0.0;
+    if (threadIdx.x < k) {
+      const unsigned long long idx = h + threadIdx.x;
+      unsigned long long* slot = self.ring + (idx & self.mask);
+      const unsigned long long want = nb_tag(idx, 0) >> 32;
+      unsigned long long x;
+      while (((x = ld_acquire(slot)) >> 32) != want) {
+        if (nb_aborted(prm.glob)) break;
+        __nanosleep(32);
+      }
+      if ((x >> 32) == want) {
+        st_relaxed(slot, 0ull);
+        const uint32_t v = (uint32_t)x;
+        // Alg.4: take the residue, add it to the rank, push alpha*rho/deg to the neighbours
+        const double rho = __longlong_as_double((long long)atomicExch((unsigned long long*)(self.res + v), 0ull));
+        start = __ldg(self.row_ptr + v);
+        deg = __ldg(self.row_ptr + v + 1) - start;
+        if (rho != 0.0) red_add_f64(self.rank + v, rho);
+        if (rho == 0.0) deg = 0;  // dangling (deg 0) absorbs (R-PR-3)
+        else if (deg) delta = prm.alpha * rho / (double)deg;
+      }
+    }
+    // warp-level load-balanced expand of this warp's 32 items
+    uint32_t incl = deg;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+      if ((int)lane >= o) incl += y;
+    }
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    s_off[wid][lane] = incl - deg;
+    s_start[wid][lane] = start;
+    s_delta[wid][lane] = delta;
+    __syncwarp();
+    for (uint32_t base = 0; base < total; base += 32) {
+      const uint32_t e = base + lane;
+      bool act = false;
+      uint32_t o = 0, lw = 0;
+      if (e < total) {
+        uint32_t j = 0;  // largest j with s_off[j] <= e
+#pragma unroll
+        for (uint32_t step = 16; step; step >>= 1)
+          if (s_off[wid][j + step] <= e) j += step;
+        const uint32_t w = __ldg(self.col + s_start[wid][j] + (e - s_off[wid][j]));
+        const double xj = s_delta[wid][j];
+        o = w / prm.B;
+        lw = w - o * prm.B;
+        const double old = atomicAdd(prm.peers[o].res + lw, xj);
+        act = old <= prm.eps && old + xj > prm.eps;  // crossing activation (R-PR-7)
+        ++edges;
+      }
+      nb_push(prm, act, o, lw);
+    }
+    __syncthreads();
+    // every push of these k items reserved its tail slot before this increment (release)
+    if (threadIdx.x == 0) {
+      __threadfence();
+      atom_add_release(&self.ctl->done, (unsigned long long)k);
+    }
+  }
+  for (int o = 16; o; o >>= 1) edges += __shfl_xor_sync(0xffffffffu, edges, o);
+  if (lane == 0 && edges) atomicAdd(&prm.glob->edges, edges);
+}
+
+// rank_out = rank / n_global (R-PR-4); residual sum into *sum.
+__global__ void k_nb_finalize(NbParams prm, double n_global, double* sum) {
+  double acc = 0.0;
+  for (uint32_t p = 0; p < prm.P; ++p) {
+    const NbPeer pe = prm.peers[p];
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < pe.n_local;
+         v += (int64_t)gridDim.x * blockDim.x) {
+      pe.rank[v] = pe.rank[v] / n_global;
+      acc += pe.res[v];
+    }
+  }
+  for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if (lane_id() == 0 && acc != 0.0) atomicAdd(sum, acc);
+}
+
+static inline uint64_t nb_pow2(uint64_t x) {
+  uint64_t c = 1;
+  while (c < x) c <<= 1;
+  return c;
+}
+
+int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, const Resolved& r,
+                       atos_stats* st) {
+  cudaStream_t s = r.stream;
+  if (g->comm) {
+    set_error("barrier_free: only loopback partitions (num_parts > 1 on one device) in this build");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  const uint32_t P = (uint32_t)g->num_parts;
+  if (P < 2 || P > kNbMaxParts) {
+    set_error("barrier_free: needs a loopback-partitioned graph with 2..%u partitions (got %u)", kNbMaxParts, P);
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  if (r.check_size > 0) {
+    set_error("barrier_free: check_size sweeps are single-partition only");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  const uint32_t B = (uint32_t)((g->n + P - 1) / P);
+  std::vector<NbPeer> peers(P);
+  for (uint32_t i = 0; i < P; ++i) {
+    Part& p = g->parts[i];
+    if (p.v_begin != (int64_t)i * B) {
+      set_error("barrier_free: partition %u does not start at %u * ceil(n/P)", i, i);
+      return ATOS_ERR_INVALID_ARG;
+    }
+    const uint64_t cap = nb_pow2((uint64_t)std::max<int64_t>(2 * p.n_local, 1024));
+    ATOS_TRY(p.nb_ring.ensure(cap * 8));
+    ATOS_TRY(p.nb_ctl.ensure(sizeof(NbCtl)));
+    ATOS_TRY(p.vbuf_a.ensure((size_t)std::max<int64_t>(p.n_local, 1) * 8));
+    ATOS_CUDA(cudaMemsetAsync(p.nb_ring.p, 0, cap * 8, s));
+    ATOS_CUDA(cudaMemsetAsync(p.nb_ctl.p, 0, sizeof(NbCtl), s));
+    p.ring_clean = false;  // conservative: the exchange-round path re-clears its own ring anyway
+    peers[i] = NbPeer{p.row_ptr, p.col, rank_out + p.v_begin, p.vbuf_a.as<double>(),
+                      p.nb_ring.as<unsigned long long>(), p.nb_ctl.as<NbCtl>(), cap - 1, (uint32_t)p.n_local, 0};
+  }
+  Part& p0 = g->parts[0];
+  const size_t tbl = sizeof(NbPeer) * P;
+  ATOS_TRY(p0.nb_peers.ensure(tbl + sizeof(NbGlob) + 64));
+  char* base = p0.nb_peers.as<char>();
+  ATOS_CUDA(cudaMemcpyAsync(base, peers.data(), tbl, cudaMemcpyHostToDevice, s));
+  NbGlob* glob = (NbGlob*)(base + tbl);
+  double* sum = (double*)(base + tbl + sizeof(NbGlob));
+  ATOS_CUDA(cudaMemsetAsync(glob, 0, sizeof(NbGlob) + 8, s));
+  NbParams prm{(const NbPeer*)base, glob, P, B, alpha, eps, r.watchdog_ns};
+  const int gs = 148 * 8;
+  k_nb_init_vertices<<<gs, 256, 0, s>>>(prm, 1.0 - alpha);
+  ++g_launches;
+  for (uint32_t i = 0; i < P; ++i) {
+    if (g->parts[i].n_local == 0) continue;
+    k_nb_init_edges<<<gs, 256, 0, s>>>(prm, i, (1.0 - alpha) * alpha);
+    ++g_launches;
+  }
+  for (uint32_t i = 0; i < P; ++i) {
+    if (g->parts[i].n_local == 0) continue;
+    k_nb_seed<<<gs, 256, 0, s>>>(prm, i);
+    ++g_launches;
+  }
+  ATOS_CUDA(cudaGetLastError());
+  int grid = 0;
+  ATOS_TRY(persistent_grid((const void*)k_pr_nobarrier, kNbBlock, 0, &grid));
+  if (r.num_blocks > 0) grid = std::min(grid, r.num_blocks);
+  grid = std::max<int>((int)P, grid - grid % (int)P);  // every partition gets the same number of CTAs
+  WorkerTimer wt;
+  wt.start(s);
+  void* args[] = {(void*)&prm};
+  ATOS_CUDA(cudaLaunchCooperativeKernel((const void*)k_pr_nobarrier, grid, kNbBlock, args, 0, s));
+  ++g_launches;
+  wt.stop(s);
+  k_nb_finalize<<<gs, 256, 0, s>>>(prm, (double)g->n, sum);
+  ++g_launches;
+  ATOS_CUDA(cudaGetLastError());
+  ATOS_TRY(stream_wait(s, r.timeout_s));
+  NbGlob hg{};
+  double hsum = 0.0;
+  ATOS_CUDA(cudaMemcpy(&hg, glob, sizeof(NbGlob), cudaMemcpyDeviceToHost));
+  ATOS_CUDA(cudaMemcpy(&hsum, sum, 8, cudaMemcpyDeviceToHost));
+  if (hg.abort) {
+    set_error("barrier_free PageRank: no progress for %.1f s (watchdog)", r.watchdog_ns * 1e-9);
+    return ATOS_ERR_TIMEOUT;
+  }
+  if (st) {
+    uint64_t pops = 0, pushes = 0;
+    for (uint32_t i = 0; i < P; ++i) {
+      NbCtl hc;
+      ATOS_CUDA(cudaMemcpy(&hc, g->parts[i].nb_ctl.p, sizeof(NbCtl), cudaMemcpyDeviceToHost));
+      pops += hc.done;
+      pushes += hc.tail;
+    }
+    st->pops += pops;
+    st->pushes += pushes;
+    st->edges += hg.edges;
+    st->rounds += 1;
+    st->residual_sum = hsum;
+    st->worker_ms += wt.elapsed();
+  }
+  return ATOS_OK;
+}
+
+}  // namespace atos

@@ -45,6 +45,9 @@ def test_cfg_layout_and_defaults():
     assert cfg.struct_size == ctypes.sizeof(_lib.Cfg)
     assert cfg.persistent == 1 and cfg.dedupe == 1 and cfg.out_where == _lib.MEM_DEVICE
     assert ctypes.sizeof(_lib.Stats) == 10 * 8 + 8 * 2
+    # barrier_free took the last reserved int: the struct keeps its size, the field is the last int
+    assert cfg.barrier_free == 0
+    assert _lib.Cfg.barrier_free.offset == _lib.Cfg.engine_variant.offset + 4
 
 
 def test_partition_range():

@@ -107,3 +107,52 @@ def test_nccl_single_rank_communicator(rmat13):
         comm.partition(g.n, 0, g.n - 1, g.row_ptr[:-1].to(DEV), g.col.to(DEV))
     part.close()
     comm.close()
+
+
+# ---- NEXT-4: barrier-free partitioned PageRank (nobarrier.cu) ----
+
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_pagerank_barrier_free_rmat(rmat13, P):
+    """One persistent kernel, remote mass straight into the owner's residue slice: same north_star bound
+    as the exchange rounds and the same conservation (no mass lost or duplicated)."""
+    g, rp, ci = rmat13
+    ref, _, _ = oracle.pagerank_jacobi(rp, ci, 0.85)
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=P)
+    for eps in (1e-6, 1e-9):
+        r, st = atos.pagerank(csr, 0.85, eps, barrier_free=1)
+        err = check_pr(rp, ci, r, st, eps, ref=ref)
+        assert abs(err) < 1e-9 * g.n, "mass lost or duplicated"
+        assert st["rounds"] == 1 and st["bytes_exchanged"] == 0
+        assert st["pops"] >= 1 and st["edges"] >= 1
+
+
+def test_pagerank_barrier_free_star_closed_form():
+    n = 5001
+    rp, ci = G.star(n)
+    csr = csr_of(rp, ci, num_parts=4)
+    r, st = atos.pagerank(csr, 0.85, 1e-10, barrier_free=1)
+    a = 0.85
+    xc = (1 + a * (n - 1)) / (1 + a)
+    xl = (1 - a) + a * xc / (n - 1)
+    x = r.cpu().numpy() * n
+    np.testing.assert_allclose(x[0], xc, rtol=1e-8)
+    np.testing.assert_allclose(x[1:], xl, rtol=1e-8)
+
+
+def test_pagerank_barrier_free_ragged_and_dangling():
+    """n not a multiple of P (short last partition), isolated and dangling vertices, host output."""
+    import torch
+    rp, ci = G.csr_from_edges(11, [(0, 1), (1, 0), (1, 2), (2, 1), (3, 4), (4, 3), (5, 6), (6, 7), (7, 5),
+                                   (8, 9)])
+    ref, _, _ = oracle.pagerank_jacobi(rp, ci, 0.85)
+    csr = csr_of(rp, ci, num_parts=3)
+    out = torch.empty(11, dtype=torch.float64)
+    r, st = atos.pagerank(csr, 0.85, 1e-12, out=out, barrier_free=1)
+    check_pr(rp, ci, r, st, 1e-12, ref=ref)
+
+
+def test_pagerank_barrier_free_unsupported(rmat13):
+    g, rp, ci = rmat13
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=1)
+    with pytest.raises(RuntimeError, match="UNSUPPORTED"):
+        atos.pagerank(csr, 0.85, 1e-6, barrier_free=1)
