@@ -11,8 +11,8 @@
 // increment, so equal sums imply a moment with nothing queued or in flight anywhere).
 //
 // Worker: a CTA claims up to 256 items of ITS partition's ring (one CAS on head, never past tail), each
-// thread begins one item (atomicExch residue -> rank, delta = alpha*rho/deg, Alg.4), and each
-// warp expands its 32 items' rows load-balanced.  Pushes are warp-aggregated per destination partition
+// thread begins one item (atomicExch residue -> rank, delta = alpha*rho/deg, Alg.4), and the
+// CTA expands the batch's rows load-balanced (block scan + search, so a hub is split over 256 threads).  Pushes are warp-aggregated per destination partition
 // (match_any + one atomicAdd on that ring's tail).  Slots carry a lap tag so a consumer never mistakes
 // the previous lap's value for its own item.
 #include "internal.h"
@@ -23,6 +23,7 @@ namespace {
 
 constexpr uint32_t kNbMaxParts = 8;
 constexpr int kNbBlock = 256;
+constexpr int kNbU = 4;  // edges in flight per lane
 
 struct NbCtl {  // one per partition; each counter on its own 128-byte line
   unsigned long long head, pad0[15];
@@ -50,6 +51,8 @@ struct NbParams {
   const NbPeer* peers;  // device array [P]
   NbGlob* glob;
   uint32_t P, B;        // partitions, block size ceil(n / P) (atos_partition_range)
+  int shift;            // log2(B) when B is a power of two, else -1
+  uint32_t S;           // sub-queues per partition (each its own ring + counters; fewer CTAs per head)
   double alpha, eps;
   unsigned long long watchdog_ns;
 };
@@ -73,12 +76,13 @@ __device__ __forceinline__ void nb_push(const NbParams& prm, bool act, uint32_t 
   const int leader = __ffs(grp) - 1;
   const uint32_t rank = __popc(grp & ((1u << lane) - 1u));
   const NbPeer* pe = prm.peers + o;
-  NbCtl* c = pe->ctl;
+  const uint32_t sub = (blockIdx.x * (blockDim.x >> 5) + warp_id()) % prm.S;  // uniform per warp
+  NbCtl* c = pe->ctl + sub;
   unsigned long long base = 0;
   if ((int)lane == leader) base = atomicAdd(&c->tail, (unsigned long long)__popc(grp));
   base = __shfl_sync(grp, base, leader);
   const unsigned long long idx = base + rank;
-  unsigned long long* slot = pe->ring + (idx & pe->mask);
+  unsigned long long* slot = pe->ring + sub * (pe->mask + 1) + (idx & pe->mask);
   // the previous lap's consumer may not have released the slot yet
   while (ld_relaxed(slot) != 0ull) {
     if (nb_aborted(prm.glob)) return;
@@ -131,34 +135,40 @@ __global__ void k_nb_seed(NbParams prm, uint32_t p) {
 
 // The persistent barrier-free worker kernel (one cooperative launch; CTA b serves partition b % P).
 // A CTA claims up to kNbBlock items of its partition's ring with ONE CAS (fewer contenders on head than
-// a claim per warp); warp w takes items [32w, 32w+32) of the batch and expands them load-balanced: a warp
-// scan of the 32 degrees, then every lane takes edge e of the batch's concatenated rows and finds its item
-// by a 5-step search over the 32 row offsets (the warp-level form of the CTA worker's LBS).
+// a claim per warp) and expands them as the paper's CTA worker with LBS does.
 __global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
   __shared__ unsigned long long s_h;
   __shared__ uint32_t s_k;
   __shared__ int s_quit;
-  __shared__ uint32_t s_off[kNbBlock / 32][32], s_start[kNbBlock / 32][32];
-  __shared__ double s_delta[kNbBlock / 32][32];
-  const uint32_t me = blockIdx.x % prm.P;
+  __shared__ uint32_t s_off[kNbBlock], s_start[kNbBlock], s_wsum[kNbBlock / 32];
+  __shared__ double s_delta[kNbBlock];
+  const uint32_t q = blockIdx.x % (prm.P * prm.S);
+  const uint32_t me = q / prm.S, sub0 = q % prm.S;
   const NbPeer self = prm.peers[me];
+  __shared__ uint32_t s_sq;
   const uint32_t lane = lane_id(), wid = warp_id();
   unsigned long long edges = 0, t_idle = 0, last_done = 0;
   while (true) {
     if (threadIdx.x == 0) {
-      uint32_t k = 0;
-      unsigned long long h = 0, hh = ld_relaxed(&self.ctl->head);
-      while (true) {
-        const unsigned long long t = ld_relaxed(&self.ctl->tail);
-        if (hh >= t) break;
-        const uint32_t want = (uint32_t)min((unsigned long long)kNbBlock, t - hh);
-        const unsigned long long got = atomicCAS(&self.ctl->head, hh, hh + want);
-        if (got == hh) {
-          h = hh;
-          k = want;
-          break;
+      uint32_t k = 0, sq = sub0;
+      unsigned long long h = 0;
+      // own sub-queue first, then the partition's other sub-queues
+      for (uint32_t i = 0; i < prm.S && k == 0; ++i) {
+        sq = (sub0 + i) % prm.S;
+        NbCtl* c = self.ctl + sq;
+        unsigned long long hh = ld_relaxed(&c->head);
+        while (true) {
+          const unsigned long long t = ld_relaxed(&c->tail);
+          if (hh >= t) break;
+          const uint32_t want = (uint32_t)min((unsigned long long)kNbBlock, t - hh);
+          const unsigned long long got = atomicCAS(&c->head, hh, hh + want);
+          if (got == hh) {
+            h = hh;
+            k = want;
+            break;
+          }
+          hh = got;
         }
-        hh = got;
       }
       int quit = 0;
       if (k == 0) {
@@ -166,8 +176,10 @@ __global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
           quit = 1;
         } else {
           unsigned long long D = 0, T = 0;
-          for (uint32_t p = 0; p < prm.P; ++p) D += atom_read(&prm.peers[p].ctl->done);
-          for (uint32_t p = 0; p < prm.P; ++p) T += atom_read(&prm.peers[p].ctl->tail);
+          for (uint32_t p = 0; p < prm.P; ++p)
+            for (uint32_t j = 0; j < prm.S; ++j) D += atom_read(&prm.peers[p].ctl[j].done);
+          for (uint32_t p = 0; p < prm.P; ++p)
+            for (uint32_t j = 0; j < prm.S; ++j) T += atom_read(&prm.peers[p].ctl[j].tail);
           if (D == T) {
             quit = 1;
           } else {
@@ -188,11 +200,13 @@ __global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
       }
       s_h = h;
       s_k = k;
+      s_sq = sq;
       s_quit = quit;
     }
     __syncthreads();
     const unsigned long long h = s_h;
     const uint32_t k = s_k;
+    const uint32_t sq = s_sq;
     const int quit = s_quit;
     __syncthreads();
     if (quit) break;
@@ -202,7 +216,7 @@ __global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
     double delta = 0.0;
     if (threadIdx.x < k) {
       const unsigned long long idx = h + threadIdx.x;
-      unsigned long long* slot = self.ring + (idx & self.mask);
+      unsigned long long* slot = self.ring + sq * (self.mask + 1) + (idx & self.mask);
       const unsigned long long want = nb_tag(idx, 0) >> 32;
       unsigned long long x;
       while (((x = ld_acquire(slot)) >> 32) != want) {
@@ -221,41 +235,59 @@ __global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
         else if (deg) delta = prm.alpha * rho / (double)deg;
       }
     }
-    // warp-level load-balanced expand of this warp's 32 items
+    // CTA-level load-balanced expand: block scan of the k degrees, then thread t takes edge
+    // e = base + u*kNbBlock + t of the batch's concatenated rows and finds its item by binary search
     uint32_t incl = deg;
     for (int o = 1; o < 32; o <<= 1) {
       const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
       if ((int)lane >= o) incl += y;
     }
-    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-    s_off[wid][lane] = incl - deg;
-    s_start[wid][lane] = start;
-    s_delta[wid][lane] = delta;
-    __syncwarp();
-    for (uint32_t base = 0; base < total; base += 32) {
-      const uint32_t e = base + lane;
-      bool act = false;
-      uint32_t o = 0, lw = 0;
-      if (e < total) {
-        uint32_t j = 0;  // largest j with s_off[j] <= e
+    if (lane == 31) s_wsum[wid] = incl;
+    __syncthreads();
+    uint32_t wbase = 0, total = 0;
 #pragma unroll
-        for (uint32_t step = 16; step; step >>= 1)
-          if (s_off[wid][j + step] <= e) j += step;
-        const uint32_t w = __ldg(self.col + s_start[wid][j] + (e - s_off[wid][j]));
-        const double xj = s_delta[wid][j];
-        o = w / prm.B;
-        lw = w - o * prm.B;
-        const double old = atomicAdd(prm.peers[o].res + lw, xj);
-        act = old <= prm.eps && old + xj > prm.eps;  // crossing activation (R-PR-7)
-        ++edges;
+    for (int w2 = 0; w2 < kNbBlock / 32; ++w2) {
+      const uint32_t x = s_wsum[w2];
+      if (w2 < (int)wid) wbase += x;
+      total += x;
+    }
+    s_off[threadIdx.x] = wbase + incl - deg;
+    s_start[threadIdx.x] = start;
+    s_delta[threadIdx.x] = delta;
+    __syncthreads();
+    for (uint32_t base = 0; base < total; base += kNbBlock * kNbU) {
+      bool act[kNbU];
+      uint32_t o[kNbU], lw[kNbU];
+#pragma unroll
+      for (int u = 0; u < kNbU; ++u) {
+        const uint32_t e = base + u * kNbBlock + threadIdx.x;
+        act[u] = false;
+        o[u] = 0;
+        lw[u] = 0;
+        if (e < total) {
+          uint32_t j = 0;  // largest j with s_off[j] <= e
+#pragma unroll
+          for (uint32_t step = kNbBlock / 2; step; step >>= 1)
+            if (s_off[j + step] <= e) j += step;
+          const uint32_t w = __ldg(self.col + s_start[j] + (e - s_off[j]));
+          const double xj = s_delta[j];
+          o[u] = prm.shift >= 0 ? (w >> prm.shift) : w / prm.B;
+          lw[u] = w - o[u] * prm.B;
+          const double old = atomicAdd(prm.peers[o[u]].res + lw[u], xj);
+          act[u] = old <= prm.eps && old + xj > prm.eps;  // crossing activation (R-PR-7)
+          ++edges;
+        }
       }
-      nb_push(prm, act, o, lw);
+#pragma unroll
+      for (int u = 0; u < kNbU; ++u) {
+        if (base + u * kNbBlock < total) nb_push(prm, act[u], o[u], lw[u]);
+      }
     }
     __syncthreads();
     // every push of these k items reserved its tail slot before this increment (release)
     if (threadIdx.x == 0) {
       __threadfence();
-      atom_add_release(&self.ctl->done, (unsigned long long)k);
+      atom_add_release(&self.ctl[sq].done, (unsigned long long)k);
     }
   }
   for (int o = 16; o; o >>= 1) edges += __shfl_xor_sync(0xffffffffu, edges, o);
@@ -300,6 +332,10 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
     return ATOS_ERR_UNSUPPORTED;
   }
   const uint32_t B = (uint32_t)((g->n + P - 1) / P);
+  // sub-queues per partition (fewer CTAs per head CAS, but shorter FIFOs pop vertices with less
+  // accumulated residue, i.e. more pops); ATOS_NB_SUBQ overrides (tools/nb_ab.py)
+  uint32_t S = P >= 4 ? 1u : 2u;
+  if (const char* e = getenv("ATOS_NB_SUBQ")) S = (uint32_t)std::max(1, std::min(16, atoi(e)));
   std::vector<NbPeer> peers(P);
   for (uint32_t i = 0; i < P; ++i) {
     Part& p = g->parts[i];
@@ -308,11 +344,11 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
       return ATOS_ERR_INVALID_ARG;
     }
     const uint64_t cap = nb_pow2((uint64_t)std::max<int64_t>(2 * p.n_local, 1024));
-    ATOS_TRY(p.nb_ring.ensure(cap * 8));
-    ATOS_TRY(p.nb_ctl.ensure(sizeof(NbCtl)));
+    ATOS_TRY(p.nb_ring.ensure(S * cap * 8));
+    ATOS_TRY(p.nb_ctl.ensure(S * sizeof(NbCtl)));
     ATOS_TRY(p.vbuf_a.ensure((size_t)std::max<int64_t>(p.n_local, 1) * 8));
-    ATOS_CUDA(cudaMemsetAsync(p.nb_ring.p, 0, cap * 8, s));
-    ATOS_CUDA(cudaMemsetAsync(p.nb_ctl.p, 0, sizeof(NbCtl), s));
+    ATOS_CUDA(cudaMemsetAsync(p.nb_ring.p, 0, S * cap * 8, s));
+    ATOS_CUDA(cudaMemsetAsync(p.nb_ctl.p, 0, S * sizeof(NbCtl), s));
     p.ring_clean = false;  // conservative: the exchange-round path re-clears its own ring anyway
     peers[i] = NbPeer{p.row_ptr, p.col, rank_out + p.v_begin, p.vbuf_a.as<double>(),
                       p.nb_ring.as<unsigned long long>(), p.nb_ctl.as<NbCtl>(), cap - 1, (uint32_t)p.n_local, 0};
@@ -325,7 +361,12 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
   NbGlob* glob = (NbGlob*)(base + tbl);
   double* sum = (double*)(base + tbl + sizeof(NbGlob));
   ATOS_CUDA(cudaMemsetAsync(glob, 0, sizeof(NbGlob) + 8, s));
-  NbParams prm{(const NbPeer*)base, glob, P, B, alpha, eps, r.watchdog_ns};
+  int shift = -1;
+  if ((B & (B - 1)) == 0) {
+    shift = 0;
+    while ((1u << shift) < B) ++shift;
+  }
+  NbParams prm{(const NbPeer*)base, glob, P, B, shift, S, alpha, eps, r.watchdog_ns};
   const int gs = 148 * 8;
   k_nb_init_vertices<<<gs, 256, 0, s>>>(prm, 1.0 - alpha);
   ++g_launches;
@@ -343,7 +384,8 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
   int grid = 0;
   ATOS_TRY(persistent_grid((const void*)k_pr_nobarrier, kNbBlock, 0, &grid));
   if (r.num_blocks > 0) grid = std::min(grid, r.num_blocks);
-  grid = std::max<int>((int)P, grid - grid % (int)P);  // every partition gets the same number of CTAs
+  const int Q = (int)(P * S);
+  grid = std::max<int>(Q, grid - grid % Q);  // every sub-queue gets the same number of CTAs
   WorkerTimer wt;
   wt.start(s);
   void* args[] = {(void*)&prm};
@@ -365,10 +407,12 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
   if (st) {
     uint64_t pops = 0, pushes = 0;
     for (uint32_t i = 0; i < P; ++i) {
-      NbCtl hc;
-      ATOS_CUDA(cudaMemcpy(&hc, g->parts[i].nb_ctl.p, sizeof(NbCtl), cudaMemcpyDeviceToHost));
-      pops += hc.done;
-      pushes += hc.tail;
+      std::vector<NbCtl> hc(S);
+      ATOS_CUDA(cudaMemcpy(hc.data(), g->parts[i].nb_ctl.p, S * sizeof(NbCtl), cudaMemcpyDeviceToHost));
+      for (uint32_t j = 0; j < S; ++j) {
+        pops += hc[j].done;
+        pushes += hc[j].tail;
+      }
     }
     st->pops += pops;
     st->pushes += pushes;
