@@ -445,6 +445,16 @@ def c5_extras(args, g, csr, sources, flush, peak):
         lres[f"bfs_P{P}"] = {"ms": float(np.mean(ms)), "rounds": int(st["rounds"]),
                              "bytes_exchanged": int(st["bytes_exchanged"]), "edges_per_m": st["edges"] / g.m,
                              "equal_to_single": bool(torch.equal(dout, ref))}
+        # NEXT-4 barrier-free protocol on the same partitions (one persistent kernel, all partitions at once)
+        atos.bfs(pc, sources[0], out=dout, barrier_free=1)
+        ms = []
+        for _ in range(2):
+            flush_l2(flush)
+            torch.cuda.synchronize()
+            _, st = atos.bfs(pc, sources[0], out=dout, barrier_free=1)
+            ms.append(st["kernel_ms"])
+        lres[f"bfs_P{P}_barrier_free"] = {"ms": float(np.mean(ms)), "edges_per_m": st["edges"] / g.m,
+                                          "equal_to_single": bool(torch.equal(dout, ref))}
         pc.close()
         torch.cuda.empty_cache()
     res["partitioned_loopback_c5"] = lres

@@ -131,10 +131,11 @@ typedef struct {
                                    48-register, 5-CTAs-per-SM build with 2 edges in flight per thread on
                                    graphs with m < 8n and 4 otherwise); 1 = the 64-register build (4 edges
                                    in flight) for every worker size */
-    int      barrier_free;      /* PageRank on a loopback-partitioned graph (num_parts 2..8): 1 = the barrier-free
-                                   protocol (NEXT-4, nobarrier.cu): one persistent kernel, remote mass and
-                                   activations go straight into the owner's residue slice and queue, global
-                                   quiescence termination; 0 (default) = exchange rounds.  ATOS_ERR_UNSUPPORTED on a
+    int      barrier_free;      /* BFS / PageRank on a loopback-partitioned graph (num_parts 2..8): 1 = the
+                                   barrier-free protocol (NEXT-4, nobarrier.cu): one persistent kernel; a remote
+                                   relaxation (BFS atomicMin on depth, PageRank atomicAdd on residue) and its
+                                   activation go straight into the owner's slice and queue; global quiescence
+                                   termination; 0 (default) = exchange rounds.  ATOS_ERR_UNSUPPORTED on a
                                    single-partition or multi-process graph */
 } atos_cfg;
 

@@ -651,7 +651,14 @@ int atos_bfs(const atos_csr* gc, int64_t src, uint32_t* depth_out, const atos_cf
   atos_stats* st = r.stats ? &local : nullptr;
   CallTimer tm(r.stream);
   int rc;
-  if (g->comm || g->num_parts > 1) {
+  if (r.barrier_free) {
+    if (g->comm || g->num_parts < 2) {
+      set_error("atos_bfs: barrier_free needs a loopback-partitioned graph (num_parts > 1, one process)");
+      return ATOS_ERR_UNSUPPORTED;
+    }
+    rc = run_with_output<uint32_t>(g, depth_out, g->n, r, g->parts[0].vbuf_c,
+                                   [&](uint32_t* d) { return bfs_nobarrier(g, src, d, r, st); });
+  } else if (g->comm || g->num_parts > 1) {
     const int64_t len = g->comm ? g->parts[0].n_local : g->n;
     rc = run_with_output<uint32_t>(g, depth_out, len, r, g->parts[0].vbuf_c,
                                    [&](uint32_t* d) { return bfs_partitioned(g, src, d, r, st); });

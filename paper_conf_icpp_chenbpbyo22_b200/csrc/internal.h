@@ -218,7 +218,8 @@ int color_count(Part& p, const int32_t* color, int64_t* used, cudaStream_t s);
 int bfs_partitioned(atos_csr* g, int64_t src, uint32_t* depth_dev, const Resolved& r, atos_stats* st);
 int pagerank_partitioned(atos_csr* g, double alpha, double eps, double* rank_dev, const Resolved& r,
                          atos_stats* st);
-// barrier-free partitioned PageRank, loopback partitions (nobarrier.cu, NEXT-4)
+// barrier-free partitioned BFS / PageRank, loopback partitions (nobarrier.cu, NEXT-4)
+int bfs_nobarrier(atos_csr* g, int64_t src, uint32_t* depth_dev, const Resolved& r, atos_stats* st);
 int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_dev, const Resolved& r,
                        atos_stats* st);
 

@@ -40,6 +40,8 @@ struct NbPeer {  // what a partition exposes to its peers (peer-mapped in a mult
   NbCtl* ctl;
   unsigned long long mask;  // cap - 1
   uint32_t n_local, pad;
+  uint32_t* depth;          // BFS: n_local (caller's output slice)
+  uint32_t* inq;            // BFS: in-queue bitmap, one bit per local vertex (dedupe)
 };
 
 struct NbGlob {
@@ -136,7 +138,8 @@ __global__ void k_nb_seed(NbParams prm, uint32_t p) {
 // The persistent barrier-free worker kernel (one cooperative launch; CTA b serves partition b % P).
 // A CTA claims up to kNbBlock items of its partition's ring with ONE CAS (fewer contenders on head than
 // a claim per warp) and expands them as the paper's CTA worker with LBS does.
-__global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
+template <bool kBfs>
+__global__ void __launch_bounds__(kNbBlock, 4) k_nobarrier(NbParams prm) {
   __shared__ unsigned long long s_h;
   __shared__ uint32_t s_k;
   __shared__ int s_quit;
@@ -226,13 +229,20 @@ __global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
       if ((x >> 32) == want) {
         st_relaxed(slot, 0ull);
         const uint32_t v = (uint32_t)x;
-        // Alg.4: take the residue, add it to the rank, push alpha*rho/deg to the neighbours
-        const double rho = __longlong_as_double((long long)atomicExch((unsigned long long*)(self.res + v), 0ull));
         start = __ldg(self.row_ptr + v);
         deg = __ldg(self.row_ptr + v + 1) - start;
-        if (rho != 0.0) red_add_f64(self.rank + v, rho);
-        if (rho == 0.0) deg = 0;  // dangling (deg 0) absorbs (R-PR-3)
-        else if (deg) delta = prm.alpha * rho / (double)deg;
+        if (kBfs) {
+          // clear the in-queue bit BEFORE reading the depth: a later improvement re-queues (SURVEY 8(a) note 3)
+          atom_and_acquire(self.inq + (v >> 5), ~(1u << (v & 31)));
+          delta = (double)(ld_relaxed(self.depth + v) + 1u);  // d + 1, exact in f64
+        } else {
+          // Alg.4: take the residue, add it to the rank, push alpha*rho/deg to the neighbours
+          const double rho =
+              __longlong_as_double((long long)atomicExch((unsigned long long*)(self.res + v), 0ull));
+          if (rho != 0.0) red_add_f64(self.rank + v, rho);
+          if (rho == 0.0) deg = 0;  // dangling (deg 0) absorbs (R-PR-3)
+          else if (deg) delta = prm.alpha * rho / (double)deg;
+        }
       }
     }
     // CTA-level load-balanced expand: block scan of the k degrees, then thread t takes edge
@@ -273,8 +283,21 @@ __global__ void __launch_bounds__(kNbBlock, 4) k_pr_nobarrier(NbParams prm) {
           const double xj = s_delta[j];
           o[u] = prm.shift >= 0 ? (w >> prm.shift) : w / prm.B;
           lw[u] = w - o[u] * prm.B;
-          const double old = atomicAdd(prm.peers[o[u]].res + lw[u], xj);
-          act[u] = old <= prm.eps && old + xj > prm.eps;  // crossing activation (R-PR-7)
+          if (kBfs) {
+            // Alg.2: atomicMin(depth[w], d+1), activate on improvement; stale-read prefilter
+            const uint32_t nd = (uint32_t)xj;
+            const NbPeer* pe = prm.peers + o[u];
+            if (ld_relaxed(pe->depth + lw[u]) > nd) {
+              const uint32_t old = atomicMin(pe->depth + lw[u], nd);
+              if (old > nd) {
+                const uint32_t bit = 1u << (lw[u] & 31);
+                act[u] = !(atom_or_release(pe->inq + (lw[u] >> 5), bit) & bit);
+              }
+            }
+          } else {
+            const double old = atomicAdd(prm.peers[o[u]].res + lw[u], xj);
+            act[u] = old <= prm.eps && old + xj > prm.eps;  // crossing activation (R-PR-7)
+          }
           ++edges;
         }
       }
@@ -315,8 +338,19 @@ static inline uint64_t nb_pow2(uint64_t x) {
   return c;
 }
 
-int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, const Resolved& r,
-                       atos_stats* st) {
+// BFS source seed: depth[src] = 0, its in-queue bit set, one push into its owner's ring.
+__global__ void k_nb_bfs_seed(NbParams prm, uint32_t o, uint32_t l) {
+  if (lane_id() == 0) {
+    prm.peers[o].depth[l] = 0u;
+    prm.peers[o].inq[l >> 5] = 1u << (l & 31);
+  }
+  __syncwarp();
+  nb_push(prm, lane_id() == 0, o, l);
+}
+
+// Shared driver: PageRank (rank_out) or BFS (depth_out, src).
+static int run_nobarrier(atos_csr* g, bool bfs, double alpha, double eps, double* rank_out, uint32_t* depth_out,
+                         int64_t src, const Resolved& r, atos_stats* st) {
   cudaStream_t s = r.stream;
   if (g->comm) {
     set_error("barrier_free: only loopback partitions (num_parts > 1 on one device) in this build");
@@ -327,14 +361,14 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
     set_error("barrier_free: needs a loopback-partitioned graph with 2..%u partitions (got %u)", kNbMaxParts, P);
     return ATOS_ERR_UNSUPPORTED;
   }
-  if (r.check_size > 0) {
+  if (!bfs && r.check_size > 0) {
     set_error("barrier_free: check_size sweeps are single-partition only");
     return ATOS_ERR_UNSUPPORTED;
   }
   const uint32_t B = (uint32_t)((g->n + P - 1) / P);
   // sub-queues per partition (fewer CTAs per head CAS, but shorter FIFOs pop vertices with less
   // accumulated residue, i.e. more pops); ATOS_NB_SUBQ overrides (tools/nb_ab.py)
-  uint32_t S = P >= 4 ? 1u : 2u;
+  uint32_t S = (bfs || P >= 4) ? 1u : 2u;
   if (const char* e = getenv("ATOS_NB_SUBQ")) S = (uint32_t)std::max(1, std::min(16, atoi(e)));
   std::vector<NbPeer> peers(P);
   for (uint32_t i = 0; i < P; ++i) {
@@ -346,12 +380,18 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
     const uint64_t cap = nb_pow2((uint64_t)std::max<int64_t>(2 * p.n_local, 1024));
     ATOS_TRY(p.nb_ring.ensure(S * cap * 8));
     ATOS_TRY(p.nb_ctl.ensure(S * sizeof(NbCtl)));
-    ATOS_TRY(p.vbuf_a.ensure((size_t)std::max<int64_t>(p.n_local, 1) * 8));
+    ATOS_TRY(p.vbuf_a.ensure((size_t)std::max<int64_t>(p.n_local, 1) * 8));  // PR residue / BFS in-queue bits
     ATOS_CUDA(cudaMemsetAsync(p.nb_ring.p, 0, S * cap * 8, s));
     ATOS_CUDA(cudaMemsetAsync(p.nb_ctl.p, 0, S * sizeof(NbCtl), s));
     p.ring_clean = false;  // conservative: the exchange-round path re-clears its own ring anyway
-    peers[i] = NbPeer{p.row_ptr, p.col, rank_out + p.v_begin, p.vbuf_a.as<double>(),
-                      p.nb_ring.as<unsigned long long>(), p.nb_ctl.as<NbCtl>(), cap - 1, (uint32_t)p.n_local, 0};
+    peers[i] = NbPeer{p.row_ptr, p.col, bfs ? nullptr : rank_out + p.v_begin, bfs ? nullptr : p.vbuf_a.as<double>(),
+                      p.nb_ring.as<unsigned long long>(), p.nb_ctl.as<NbCtl>(), cap - 1, (uint32_t)p.n_local, 0,
+                      bfs ? depth_out + p.v_begin : nullptr, bfs ? p.vbuf_a.as<uint32_t>() : nullptr};
+    if (bfs) {
+      // Alg.1 init P:721-725: depth = MAX_UINT32, nothing queued
+      if (p.n_local) ATOS_CUDA(cudaMemsetAsync(depth_out + p.v_begin, 0xFF, (size_t)p.n_local * 4, s));
+      ATOS_CUDA(cudaMemsetAsync(p.vbuf_a.p, 0, ((size_t)p.n_local / 32 + 1) * 4, s));
+    }
   }
   Part& p0 = g->parts[0];
   const size_t tbl = sizeof(NbPeer) * P;
@@ -368,32 +408,41 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
   }
   NbParams prm{(const NbPeer*)base, glob, P, B, shift, S, alpha, eps, r.watchdog_ns};
   const int gs = 148 * 8;
-  k_nb_init_vertices<<<gs, 256, 0, s>>>(prm, 1.0 - alpha);
-  ++g_launches;
-  for (uint32_t i = 0; i < P; ++i) {
-    if (g->parts[i].n_local == 0) continue;
-    k_nb_init_edges<<<gs, 256, 0, s>>>(prm, i, (1.0 - alpha) * alpha);
+  if (bfs) {
+    const uint32_t o = (uint32_t)(src / B);
+    k_nb_bfs_seed<<<1, 32, 0, s>>>(prm, o, (uint32_t)(src - (int64_t)o * B));
     ++g_launches;
-  }
-  for (uint32_t i = 0; i < P; ++i) {
-    if (g->parts[i].n_local == 0) continue;
-    k_nb_seed<<<gs, 256, 0, s>>>(prm, i);
+  } else {
+    k_nb_init_vertices<<<gs, 256, 0, s>>>(prm, 1.0 - alpha);
     ++g_launches;
+    for (uint32_t i = 0; i < P; ++i) {
+      if (g->parts[i].n_local == 0) continue;
+      k_nb_init_edges<<<gs, 256, 0, s>>>(prm, i, (1.0 - alpha) * alpha);
+      ++g_launches;
+    }
+    for (uint32_t i = 0; i < P; ++i) {
+      if (g->parts[i].n_local == 0) continue;
+      k_nb_seed<<<gs, 256, 0, s>>>(prm, i);
+      ++g_launches;
+    }
   }
   ATOS_CUDA(cudaGetLastError());
   int grid = 0;
-  ATOS_TRY(persistent_grid((const void*)k_pr_nobarrier, kNbBlock, 0, &grid));
+  const void* fn = bfs ? (const void*)k_nobarrier<true> : (const void*)k_nobarrier<false>;
+  ATOS_TRY(persistent_grid(fn, kNbBlock, 0, &grid));
   if (r.num_blocks > 0) grid = std::min(grid, r.num_blocks);
   const int Q = (int)(P * S);
   grid = std::max<int>(Q, grid - grid % Q);  // every sub-queue gets the same number of CTAs
   WorkerTimer wt;
   wt.start(s);
   void* args[] = {(void*)&prm};
-  ATOS_CUDA(cudaLaunchCooperativeKernel((const void*)k_pr_nobarrier, grid, kNbBlock, args, 0, s));
+  ATOS_CUDA(cudaLaunchCooperativeKernel(fn, grid, kNbBlock, args, 0, s));
   ++g_launches;
   wt.stop(s);
-  k_nb_finalize<<<gs, 256, 0, s>>>(prm, (double)g->n, sum);
-  ++g_launches;
+  if (!bfs) {
+    k_nb_finalize<<<gs, 256, 0, s>>>(prm, (double)g->n, sum);
+    ++g_launches;
+  }
   ATOS_CUDA(cudaGetLastError());
   ATOS_TRY(stream_wait(s, r.timeout_s));
   NbGlob hg{};
@@ -401,7 +450,7 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
   ATOS_CUDA(cudaMemcpy(&hg, glob, sizeof(NbGlob), cudaMemcpyDeviceToHost));
   ATOS_CUDA(cudaMemcpy(&hsum, sum, 8, cudaMemcpyDeviceToHost));
   if (hg.abort) {
-    set_error("barrier_free PageRank: no progress for %.1f s (watchdog)", r.watchdog_ns * 1e-9);
+    set_error("barrier_free %s: no progress for %.1f s (watchdog)", bfs ? "BFS" : "PageRank", r.watchdog_ns * 1e-9);
     return ATOS_ERR_TIMEOUT;
   }
   if (st) {
@@ -418,10 +467,20 @@ int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, 
     st->pushes += pushes;
     st->edges += hg.edges;
     st->rounds += 1;
-    st->residual_sum = hsum;
+    if (!bfs) st->residual_sum = hsum;
     st->worker_ms += wt.elapsed();
   }
   return ATOS_OK;
+}
+
+
+int pagerank_nobarrier(atos_csr* g, double alpha, double eps, double* rank_out, const Resolved& r,
+                       atos_stats* st) {
+  return run_nobarrier(g, false, alpha, eps, rank_out, nullptr, 0, r, st);
+}
+
+int bfs_nobarrier(atos_csr* g, int64_t src, uint32_t* depth_out, const Resolved& r, atos_stats* st) {
+  return run_nobarrier(g, true, 0.0, 0.0, nullptr, depth_out, src, r, st);
 }
 
 }  // namespace atos

@@ -151,8 +151,42 @@ def test_pagerank_barrier_free_ragged_and_dangling():
     check_pr(rp, ci, r, st, 1e-12, ref=ref)
 
 
-def test_pagerank_barrier_free_unsupported(rmat13):
+def test_barrier_free_unsupported(rmat13):
     g, rp, ci = rmat13
     csr = atos.CSR.from_graph(g.to(DEV), num_parts=1)
     with pytest.raises(RuntimeError, match="UNSUPPORTED"):
         atos.pagerank(csr, 0.85, 1e-6, barrier_free=1)
+    with pytest.raises(RuntimeError, match="UNSUPPORTED"):
+        atos.bfs(csr, 0, barrier_free=1)
+
+
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_bfs_barrier_free_rmat(rmat13, P):
+    """Barrier-free BFS over loopback partitions: remote atomicMin straight into the owner's depth slice,
+    in-queue bit dedupe; label-correcting, so bit-exact against the oracle."""
+    g, rp, ci = rmat13
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=P)
+    for s in (gen.pick_source(g, 1), 0, g.n - 1):
+        d, st = atos.bfs(csr, s, barrier_free=1)
+        np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, s))
+        assert st["rounds"] == 1 and st["bytes_exchanged"] == 0
+
+
+@pytest.mark.parametrize("P", [2, 5])
+def test_bfs_barrier_free_mesh(P):
+    R, C = 120, 97
+    g = gen.mesh(R, C)
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=P)
+    r, c = np.divmod(np.arange(R * C), C)
+    for (r0, c0) in ((0, 0), (R // 2, C // 2)):
+        d, st = atos.bfs(csr, r0 * C + c0, barrier_free=1)
+        np.testing.assert_array_equal(as_u32(d), np.abs(r - r0) + np.abs(c - c0))
+
+
+def test_bfs_barrier_free_directed_host_output():
+    import torch
+    rp, ci = G.csr_from_edges(7, [(0, 1), (1, 2), (2, 3), (3, 4), (4, 5), (5, 6), (6, 0)])
+    csr = csr_of(rp, ci, num_parts=3)
+    out = torch.empty(7, dtype=torch.int32)
+    d, st = atos.bfs(csr, 4, out=out, barrier_free=1)
+    np.testing.assert_array_equal(d.numpy().view(np.uint32), oracle.bfs(rp, ci, 4))

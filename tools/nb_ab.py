@@ -30,6 +30,13 @@ def main():
             print(f"P={P} {'barrier_free' if bf else 'rounds      '}: {st['kernel_ms']:8.1f} ms  worker "
                   f"{st['worker_ms']:8.1f} ms  edges/m {st['edges'] / g.m:6.1f}  pops/n {st['pops'] / g.n:5.1f}  "
                   f"rounds {st['rounds']}  l1 {l1:.2e}", flush=True)
+        src = gen.pick_source(g, 105)
+        for bf in (0, 1):
+            for _ in range(2):
+                d, st = atos.bfs(pc, src, barrier_free=bf)
+            torch.cuda.synchronize()
+            print(f"P={P} BFS {'barrier_free' if bf else 'rounds      '}: {st['kernel_ms']:8.2f} ms  edges/m "
+                  f"{st['edges'] / g.m:5.2f}  rounds {st['rounds']}", flush=True)
         pc.close()
 
 
