@@ -14,15 +14,18 @@ from paper_conf_icpp_chenbpbyo22_b200 import gen  # noqa: E402
 
 def main():
     scale = int(sys.argv[1]) if len(sys.argv) > 1 else 22
+    bfs_only = len(sys.argv) > 2 and sys.argv[2] == "bfs"
     g = gen.rmat(scale, 16, 3, device="cuda")
     one = atos.CSR.from_graph(g)
-    ref, st = atos.pagerank(one, 0.85, 1e-6)
-    ref, st = atos.pagerank(one, 0.85, 1e-6)
-    print(f"single: {st['kernel_ms']:.1f} ms edges/m {st['edges'] / g.m:.1f} pops/n {st['pops'] / g.n:.1f}", flush=True)
+    if not bfs_only:
+        ref, st = atos.pagerank(one, 0.85, 1e-6)
+        ref, st = atos.pagerank(one, 0.85, 1e-6)
+        print(f"single: {st['kernel_ms']:.1f} ms edges/m {st['edges'] / g.m:.1f} pops/n {st['pops'] / g.n:.1f}",
+              flush=True)
     one.close()
     for P in (2, 4, 8):
         pc = atos.CSR.from_graph(g, num_parts=P)
-        for bf in (0, 1):
+        for bf in (() if bfs_only else (0, 1)):
             for _ in range(2):
                 r, st = atos.pagerank(pc, 0.85, 1e-6, barrier_free=bf)
             torch.cuda.synchronize()
