@@ -368,7 +368,9 @@ static int run_nobarrier(atos_csr* g, bool bfs, double alpha, double eps, double
   const uint32_t B = (uint32_t)((g->n + P - 1) / P);
   // sub-queues per partition (fewer CTAs per head CAS, but shorter FIFOs pop vertices with less
   // accumulated residue, i.e. more pops); ATOS_NB_SUBQ overrides (tools/nb_ab.py)
-  uint32_t S = (bfs || P >= 4) ? 1u : 2u;
+  // measured (tools/nb_ab.py, profiles/r01_nobarrier_*subq*): PageRank C3 best at S = 2 for P = 2 and S = 1 for
+  // P >= 4 (more sub-queues add pops); BFS C5 best at S = 4 for every P (P=2 82 -> 52 ms, no added work)
+  uint32_t S = bfs ? 4u : (P >= 4 ? 1u : 2u);
   if (const char* e = getenv("ATOS_NB_SUBQ")) S = (uint32_t)std::max(1, std::min(16, atoi(e)));
   std::vector<NbPeer> peers(P);
   for (uint32_t i = 0; i < P; ++i) {
