@@ -1,4 +1,4 @@
-// nobarrier.cu -- NEXT-4: barrier-free partitioned PageRank.
+// nobarrier.cu -- NEXT-4: barrier-free partitioned PageRank and BFS.
 //
 // The exchange-round path (relax.cu pagerank_partitioned) runs every partition to local
 // quiescence, then exchanges ghost mass and starts the next round.  Here the barrier goes away, which is
@@ -10,11 +10,15 @@
 // counter and then every tail counter (monotone counters; an item's pushes are reserved before its done
 // increment, so equal sums imply a moment with nothing queued or in flight anywhere).
 //
-// Worker: a CTA claims up to 256 items of ITS partition's ring (one CAS on head, never past tail), each
-// thread begins one item (atomicExch residue -> rank, delta = alpha*rho/deg, Alg.4), and the
-// CTA expands the batch's rows load-balanced (block scan + search, so a hub is split over 256 threads).  Pushes are warp-aggregated per destination partition
-// (match_any + one atomicAdd on that ring's tail).  Slots carry a lap tag so a consumer never mistakes
-// the previous lap's value for its own item.
+// BFS runs the same kernel with Alg.2's relax: atomicMin on the owner's depth slice, activation
+// on improvement gated by the owner's in-queue bit (cleared by the popper before it reads the depth).
+//
+// Worker: a CTA claims up to 256 items of one of its partition's S sub-queue rings (one CAS on head,
+// never past tail), each thread begins one item (atomicExch residue -> rank, delta = alpha*rho/deg,
+// Alg.4), and the CTA expands the batch's rows load-balanced (block scan + search, so a hub is
+// split over 256 threads).  Pushes are warp-aggregated per destination partition (match_any + one
+// atomicAdd on that sub-queue's tail).  Slots carry a lap tag so a consumer never mistakes the previous
+// lap's value for its own item.
 #include "internal.h"
 
 namespace atos {
