@@ -28,6 +28,9 @@ namespace {
 constexpr uint32_t kNbMaxParts = 8;
 constexpr int kNbBlock = 256;
 constexpr int kNbU = 4;  // edges in flight per lane
+#ifndef ATOS_NB_MINB
+#define ATOS_NB_MINB 4  // CTAs per SM the register budget is sized for (64 registers)
+#endif
 
 struct NbCtl {  // one per partition; each counter on its own 128-byte line
   unsigned long long head, pad0[15];
@@ -143,7 +146,7 @@ __global__ void k_nb_seed(NbParams prm, uint32_t p) {
 // A CTA claims up to kNbBlock items of its partition's ring with ONE CAS (fewer contenders on head than
 // a claim per warp) and expands them as the paper's CTA worker with LBS does.
 template <bool kBfs>
-__global__ void __launch_bounds__(kNbBlock, 4) k_nobarrier(NbParams prm) {
+__global__ void __launch_bounds__(kNbBlock, ATOS_NB_MINB) k_nobarrier(NbParams prm) {
   __shared__ unsigned long long s_h;
   __shared__ uint32_t s_k;
   __shared__ int s_quit;
