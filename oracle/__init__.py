@@ -50,6 +50,8 @@ def _load():
             lib.oracle_pagerank_jacobi.restype = i32
             lib.oracle_pagerank_push.argtypes = [i64, P, P, dbl, dbl, P, P, P]
             lib.oracle_pagerank_push.restype = i32
+            lib.oracle_pagerank_residual.argtypes = [i64, P, P, dbl, P, P]
+            lib.oracle_pagerank_residual.restype = i32
             lib.oracle_color_greedy.argtypes = [i64, P, P, P, P]
             lib.oracle_color_greedy.restype = i64
             lib.oracle_color_jp.argtypes = [i64, P, P, u64, P]
@@ -115,6 +117,18 @@ def pagerank_push(row_ptr, col, alpha: float = 0.85, eps: float = 1e-6):
     if rc != 0:
         raise ValueError("oracle_pagerank_push: bad arguments")
     return out, res, int(pops.value)
+
+
+def pagerank_residual(row_ptr, col, x, alpha: float = 0.85) -> np.ndarray:
+    """r = (1-a)1 + a P^T x - x for an UNNORMALISED candidate x (x = rank * n). See oracle_pagerank_residual."""
+    n, rp, ci = _csr(row_ptr, col)
+    xx = np.ascontiguousarray(x, dtype=np.float64)
+    if xx.shape[0] != n:
+        raise ValueError("pagerank_residual: x must have n entries")
+    r = np.empty(n, dtype=np.float64)
+    if _load().oracle_pagerank_residual(n, _p(rp), _p(ci), float(alpha), _p(xx), _p(r)) != 0:
+        raise ValueError("oracle_pagerank_residual: bad arguments")
+    return r
 
 
 def color_greedy(row_ptr, col, order=None):

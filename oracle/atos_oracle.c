@@ -18,7 +18,9 @@
  * Pins (tests/test_oracle_*.py): Floyd-Warshall, closed forms (path, cycle,
  * star, complete, grid, regular graphs, star PageRank), dense LU solve,
  * brute-force chromatic numbers, hand-solved 3-vertex PageRank, JP literal
- * round simulation == JP-by-priority greedy.  The colour-count of the GPU
+ * round simulation == JP-by-priority greedy; the PageRank residual against
+ * hand values (tests/golden/pr_residual_3vertex.json), the star closed form,
+ * the dense matrix, and the push oracle's own residue array.  The colour-count of the GPU
  * path is "parity unpinned" (any proper colouring is correct).
  */
 #include <stdint.h>
@@ -209,6 +211,43 @@ int oracle_pagerank_push(int64_t n, const int64_t *row_ptr, const int32_t *col,
     if (residue_out) for (int64_t v = 0; v < n; ++v) residue_out[v] = res[v];
     if (pops_out) *pops_out = pops;
     free(rank); free(res); free(q); free(inq);
+    return 0;
+}
+
+/*
+ * PageRank residual of a candidate x (R-PR-1 definition, written out):
+ *   r_w = (1-alpha) + alpha * sum_{v->w} x_v / deg(v)  -  x_w
+ * one pass over the CSR rows, dangling rows contributing nothing (R-PR-3).
+ * This is the residue of Alg.4 as a function of the ranks alone:
+ * the push iteration keeps x* = x + (I - alpha P^T)^{-1} r at every step, and
+ * stops when every residue <= eps.  So a candidate x whose
+ * residual satisfies 0 <= r <= eps elementwise obeys
+ *   0 <= x_star - x <= eps x_star / (1-alpha)
+ * (because (I - alpha P^T)^{-1} >= 0 and (I - alpha P^T)^{-1} 1 = x_star / (1-alpha))
+ * without solving for x*: one SpMV certifies the north-star tolerance at a
+ * size where Jacobi to 1e-13 would take ~185 sweeps.  The in-neighbour sums
+ * are accumulated in long double (x87 extended, 64-bit mantissa) so the
+ * certificate's own rounding (<= indeg * 2^-64 * sum) stays far below eps
+ * even at in-degrees of 10^6; the final subtraction is rounded to double.
+ * x[n] is the UNNORMALISED rank (x = rank_out * n).  Returns 0 / -1.
+ */
+int oracle_pagerank_residual(int64_t n, const int64_t *row_ptr, const int32_t *col,
+                             double alpha, const double *x, double *r_out)
+{
+    if (n < 0 || !(alpha > 0.0 && alpha < 1.0) || !x || !r_out) return -1;
+    if (n == 0) return 0;
+    long double *y = (long double *)malloc(sizeof(long double) * (size_t)n);
+    if (!y) return -1;
+    for (int64_t w = 0; w < n; ++w) y[w] = 0.0L;
+    for (int64_t v = 0; v < n; ++v) {
+        int64_t deg = row_ptr[v + 1] - row_ptr[v];
+        if (deg == 0) continue;                        /* dangling: zero row */
+        long double share = (long double)x[v] / (long double)deg;
+        for (int64_t e = row_ptr[v]; e < row_ptr[v + 1]; ++e) y[col[e]] += share;
+    }
+    for (int64_t w = 0; w < n; ++w)
+        r_out[w] = (double)((1.0L - (long double)alpha) + (long double)alpha * y[w] - (long double)x[w]);
+    free(y);
     return 0;
 }
 

@@ -124,3 +124,69 @@ def test_bad_args():
         oracle.pagerank_jacobi(rp, ci, 1.5)
     with pytest.raises(ValueError):
         oracle.pagerank_push(rp, ci, 0.85, 0.0)
+
+
+# ---- oracle.pagerank_residual: r = (1-a)1 + a P^T x - x (the certificate used at C5 size) ----------
+
+def test_residual_golden_hand_values():
+    g = json.load(open(os.path.join(GOLD, "pr_residual_3vertex.json")))
+    rp, ci = G.csr_from_edges(g["n"], g["edges"])
+    r = oracle.pagerank_residual(rp, ci, g["x"], g["alpha"])
+    np.testing.assert_allclose(r, g["r"], rtol=0, atol=1e-15)
+
+
+def test_residual_zero_at_golden_fixed_point():
+    g = json.load(open(os.path.join(GOLD, "pr_3vertex_dangling.json")))
+    rp, ci = G.csr_from_edges(g["n"], g["edges"])
+    r = oracle.pagerank_residual(rp, ci, g["x"], g["alpha"])
+    np.testing.assert_allclose(r, 0.0, atol=1e-15)
+
+
+@pytest.mark.parametrize("n", [3, 11, 200])
+def test_residual_star_closed_form(n):
+    """Star at x = 1: centre r = (1-a) + a(n-1) - 1 = a(n-2); leaf r = (1-a) + a/(n-1) - 1."""
+    rp, ci = G.star(n)
+    r = oracle.pagerank_residual(rp, ci, np.ones(n), A)
+    np.testing.assert_allclose(r[0], A * (n - 2), rtol=1e-14)
+    np.testing.assert_allclose(r[1:], A / (n - 1) - A, rtol=1e-13)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_residual_vs_dense_and_push(seed):
+    """Against the dense matrix (multi-edges, self loops, dangling rows) at a random x; at the LU
+    solution r = 0; and the push oracle's own residue array equals the residual of its ranks
+    (the invariant x* = x + (I - a P^T)^{-1} r that the GPU certificate relies on)."""
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(20, 150))
+    m = int(n * rng.uniform(1.0, 4.0))
+    rp, ci = G.csr_from_edges(n, zip(rng.integers(0, n, m), rng.integers(0, n, m)), dedupe=False,
+                              keep_self_loops=True)
+    Adj = G.to_dense(rp, ci)
+    deg = Adj.sum(axis=1)
+    P = np.zeros_like(Adj)
+    P[deg > 0] = Adj[deg > 0] / deg[deg > 0, None]
+    x = rng.uniform(0.1, 3.0, n)
+    want = (1 - A) + A * (P.T @ x) - x
+    np.testing.assert_allclose(oracle.pagerank_residual(rp, ci, x, A), want, rtol=1e-12, atol=1e-13)
+    xs = dense_solve(rp, ci)
+    assert np.max(np.abs(oracle.pagerank_residual(rp, ci, xs, A))) < 1e-12
+    p, res, pops = oracle.pagerank_push(rp, ci, A, 1e-6)
+    np.testing.assert_allclose(oracle.pagerank_residual(rp, ci, p * n, A), res, rtol=0, atol=1e-12)
+
+
+def test_residual_at_jacobi_result_is_below_tol():
+    """Jacobi stops when |x^{k+1}-x^k|_inf <= tol; its last increment is the residual of x^k, and the residual of
+    x^{k+1} is a P^T of that increment -- so 0 <= r <= tol elementwise (monotone iterates, R-PR-oracle)."""
+    rp, ci = G.gnp(300, 0.03, seed=5)
+    for tol in (1e-4, 1e-8):
+        r_, it, ok = oracle.pagerank_jacobi(rp, ci, A, tol=tol)
+        r = oracle.pagerank_residual(rp, ci, r_ * 300, A)
+        assert np.all(r >= -1e-13) and np.all(r <= tol + 1e-13)
+
+
+def test_residual_bad_args():
+    rp, ci = G.cycle(5)
+    with pytest.raises(ValueError):
+        oracle.pagerank_residual(rp, ci, np.ones(4), A)
+    with pytest.raises(ValueError):
+        oracle.pagerank_residual(rp, ci, np.ones(5), 1.0)
