@@ -11,8 +11,13 @@ PageRank (C3) and colouring (C4) ms-to-converge are reported alongside under
 "apps" (rank 0, N = 1).  Rank 0 prints one JSON line.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl atos|reference]
-                  [--scale S] [--no-apps] [--full]
+                  [--scale S] [--no-apps] [--dry-run]
 
+--gpus N > 1 without a torchrun environment re-launches itself under
+torch.distributed.run with N ranks (one process per GPU, NCCL).  Each rank
+generates only its own 1D row block of the graph (gen.rmat(rows=...)).
+--dry-run (CPU, gloo) stops after the per-rank graph construction and source
+choice (tests/test_dist_gloo.py).
 --impl reference runs the paper-method oracle (oracle/, serial C) on the same
 workload on the host cores (rank 0 only).
 """
@@ -135,24 +140,48 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(rows)}
 
 
-def dist_setup():
+def relaunch_under_torchrun(args) -> int:
+    """--gpus N > 1 outside torchrun: run this script under torch.distributed.run with N ranks."""
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    log("[bench] relaunch:", " ".join(cmd))
+    return subprocess.call(cmd)
+
+
+def dist_setup(args):
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if ws > 1:
         import torch.distributed as dist
+        if ws != args.gpus:
+            raise SystemExit(f"[bench] WORLD_SIZE={ws} but --gpus {args.gpus}")
+        if args.dry_run:
+            dist.init_process_group("gloo")
+            return ws, rank, local
+        os.environ.setdefault("NCCL_DEBUG", "INFO")  # init lines let the driver count the ranks
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
-    else:
+    elif not args.dry_run:
         torch.cuda.set_device(local)
     return ws, rank, local
+
+
+def _coll_device():
+    import torch.distributed as dist
+    return "cuda" if dist.get_backend() == "nccl" else "cpu"
 
 
 def allreduce_max(x: float, ws: int) -> float:
     if ws == 1:
         return x
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    t = torch.tensor([x], dtype=torch.float64, device=_coll_device())
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -161,9 +190,37 @@ def allreduce_sum(x: float, ws: int) -> float:
     if ws == 1:
         return x
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    t = torch.tensor([x], dtype=torch.float64, device=_coll_device())
     dist.all_reduce(t, op=dist.ReduceOp.SUM)
     return float(t.item())
+
+
+def global_degrees(deg_local: torch.Tensor, n: int, ws: int) -> torch.Tensor:
+    """The global degree vector from the ranks' row blocks (blocks of ceil(n/ws), the last padded)."""
+    if ws == 1:
+        return deg_local
+    import torch.distributed as dist
+    chunk = (n + ws - 1) // ws
+    pad = torch.zeros(chunk, dtype=torch.int64, device=deg_local.device)
+    pad[:deg_local.numel()] = deg_local
+    out = torch.empty(chunk * ws, dtype=torch.int64, device=deg_local.device)
+    dist.all_gather_into_tensor(out, pad)
+    return out[:n]
+
+
+def make_local_graph(scale, ef, seed, device, ws, rank):
+    """This rank's 1D row block [v_begin, v_end) of the RMAT graph (the whole graph at ws = 1)."""
+    from paper_conf_icpp_chenbpbyo22_b200 import dist_host, gen
+    t = time.time()
+    n = 1 << scale
+    vb, ve = dist_host.block_range(n, ws, rank)
+    g = gen.rmat(scale, ef, seed, device=device, rows=None if ws == 1 else (vb, ve),
+                 name=f"rmat-s{scale}-ef{ef}-seed{seed}")
+    if str(device).startswith("cuda"):
+        torch.cuda.synchronize()
+    log(f"[bench] rank {rank}: rows [{vb}, {ve}) of rmat-s{scale}-ef{ef}-seed{seed}: m_local={g.m} "
+        f"in {time.time() - t:.1f}s")
+    return g, vb, ve
 
 
 def barrier(ws):
@@ -172,6 +229,19 @@ def barrier(ws):
         import torch.distributed as dist
         dist.barrier()
     torch.cuda.synchronize()
+
+
+def host_identity():
+    """The box's host CPU (record the CPU model and core count next to the oracle time)."""
+    model = "?"
+    try:
+        for l in open("/proc/cpuinfo"):
+            if l.startswith("model name"):
+                model = l.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"host_nproc": os.cpu_count(), "host_cpu_model": model}
 
 
 def flush_l2(buf):
@@ -226,7 +296,7 @@ def run_reference(args, ws, rank):
                                f"8 seeded sources, 1D vertex partition over {ws} GPU(s)",
                    "global_batch": 1, "parallelism": f"vertex-partition{ws}",
                    "implementation": "serial CPU oracle (oracle/atos_oracle.c, gcc -O2), 1 host core"},
-        "cpu_baseline": {"value": value, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+        "cpu_baseline": {"value": value, "unit": "GTEPS", "cores": 1, "kind": "oracle", **host_identity(),
                          "sample": f"full serial FIFO BFS (oracle_bfs) from each seeded source, {args.steps} steps"},
         "e2e": {"value": value, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -237,11 +307,20 @@ def run_reference(args, ws, rank):
 def run_atos(args, ws, rank, local):
     import paper_conf_icpp_chenbpbyo22_b200 as atos
     from paper_conf_icpp_chenbpbyo22_b200 import gen
-    dev = torch.device(f"cuda:{local}")
+    dev = torch.device("cpu") if args.dry_run else torch.device(f"cuda:{local}")
     peak, peak_kind = measured_peaks()
-    g = make_graph(args.scale, 16, 5, dev)
-    sources = [gen.pick_source(g, 105 + i) for i in range(8)]
+    g, vb, ve = make_local_graph(args.scale, 16, 5, dev, ws, rank)
+    deg_local = g.degrees()
+    deg_all = global_degrees(deg_local, g.n, ws)
+    sources = [gen.pick_source_from_degrees(deg_all, 105 + i) for i in range(8)]
+    del deg_all
+    if args.dry_run:
+        line = {"dry_run": True, "rank": rank, "world_size": ws, "n": g.n, "v_begin": vb, "v_end": ve,
+                "m_local": g.m, "m_total": int(allreduce_sum(float(g.m), ws)), "sources": sources}
+        print(json.dumps(line), flush=True)
+        return
     knobs = dict(worker=args.worker, fetch_size=args.fetch)
+    comm_ok = True
     if ws == 1:
         csr = atos.CSR.from_graph(g, device=local)
     else:
@@ -250,14 +329,11 @@ def run_atos(args, ws, rank, local):
         obj = [uid]
         dist.broadcast_object_list(obj, src=0)
         comm = atos.Comm(ws, rank, obj[0], local)
-        from paper_conf_icpp_chenbpbyo22_b200 import dist_host
-        vb, ve = dist_host.block_range(g.n, ws, rank)
-        rp, ci = dist_host.local_rows(g.row_ptr, g.col, vb, ve)
-        csr = comm.partition(g.n, vb, ve, rp, ci)
+        csr = comm.partition(g.n, vb, ve, g.row_ptr, g.col)
+        comm_ok = int(allreduce_sum(1.0, ws)) == ws
     # per-source reached vertices / edges (global) for GTEPS and algorithmic bytes
     out = torch.empty(csr.n_local if ws > 1 else g.n, dtype=torch.int32, device=dev)
     src_info = []
-    deg_local = g.degrees() if ws == 1 else (g.degrees()[vb:ve])
     for s in sources:
         d, st = atos.bfs(csr, s, out=out, **knobs)
         reached = d != -1
@@ -305,21 +381,26 @@ def run_atos(args, ws, rank, local):
         roofline["pattern_roofline"] = {"bound": "l1tex random-gather wavefronts (1 per edge)", "achieved": ach,
                                         "peak": gpk, "unit": "edges/s", "frac": ach / gpk,
                                         "peak_source": "profiles/r01_micro_peaks.json"}
+    m_total = int(allreduce_sum(float(g.m), ws))
     line = {
         "metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": ws, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak" if ws == 1 else "strong",
         "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-        "config": {"workload": f"C5: BFS on RMAT scale {args.scale} ef 16 seed 5 (n={g.n}, m={g.m}), "
+        "config": {"workload": f"C5: BFS on RMAT scale {args.scale} ef 16 seed 5 (n={g.n}, m={m_total}), "
                                f"8 seeded sources, 1D vertex partition over {ws} GPU(s)",
                    "global_batch": 1, "parallelism": f"vertex-partition{ws}", "worker": args.worker,
                    "fetch_size": args.fetch, "l2": "flushed (512 MiB write) before every timed step",
                    "mean_reached_vertices": float(np.mean(verts)), "mean_reached_edges": float(np.mean(edges))},
         "roofline": roofline, "clocks": clocks, "gpu_launches": int(launches),
     }
+    if ws > 1:
+        line["comm_nranks_ok"] = comm_ok
+        line["config"]["m_local_max_over_mean"] = allreduce_max(float(g.m), ws) / (m_total / ws)
     if ws == 1 and not args.no_bsp:
         line["bsp"] = {"bfs_c5": bsp_bfs(csr, sources, src_info, out, flush, ms_per_step)}
+    e2e = e2e_bfs(args, g, vb, ve, sources, src_info, knobs, local, ws, comm if ws > 1 else None)
     if rank == 0 and ws == 1:
-        line["e2e"] = e2e_bfs(args, g, sources, src_info, knobs, local)
+        line["e2e"] = e2e
         if not args.no_cpu:
             line["cpu_baseline"] = cpu_baseline(g, sources, src_info)
         if not args.no_apps:
@@ -328,7 +409,7 @@ def run_atos(args, ws, rank, local):
             torch.cuda.empty_cache()
             line["apps"].update(run_apps(args, dev, peak))
     elif rank == 0:
-        line["e2e"] = None
+        line["e2e"] = e2e
     if rank == 0:
         print(json.dumps(line), flush=True)
 
@@ -351,38 +432,49 @@ def bsp_bfs(csr, sources, src_info, out, flush, atos_ms):
             "atos_speedup": m / atos_ms, "note": "Alg.1 level-synchronous, edge-balanced advance + host barrier per level"}
 
 
-def e2e_bfs(args, g, sources, src_info, knobs, local, steps=5):
-    """Same metric through the public API with HOST buffers: pinned host CSR -> atos_csr_create
-    (H2D inside the timed region) -> atos_bfs with a host output (D2H) -> destroy.  One untimed
-    warm-up step first (first-touch of the pinned pages and of the device allocations)."""
+def e2e_bfs(args, g, vb, ve, sources, src_info, knobs, local, ws, comm):
+    """Same metric through the public API with HOST buffers, every step (args.steps of them, the
+    driver's K): pinned host CSR (this rank's rows at N > 1) -> atos_csr_create / atos_csr_create_part
+    (H2D inside the timed region) -> atos_bfs with a host output (D2H) -> destroy.  One untimed warm-up
+    step first (first touch of the pinned pages).  Wall clock per step, max over ranks, with barriers."""
     import paper_conf_icpp_chenbpbyo22_b200 as atos
     rp_h = torch.empty(g.row_ptr.shape, dtype=g.row_ptr.dtype).pin_memory()
     ci_h = torch.empty(g.col.shape, dtype=g.col.dtype).pin_memory()
     rp_h.copy_(g.row_ptr)
     ci_h.copy_(g.col)
-    out_h = torch.empty(g.n, dtype=torch.int32).pin_memory()
+    out_h = torch.empty(ve - vb, dtype=torch.int32).pin_memory()
     torch.cuda.synchronize()
-    csr = atos.CSR(rp_h, ci_h, device=local)
+
+    def create():
+        if comm is None:
+            return atos.CSR(rp_h, ci_h, device=local)
+        return comm.partition(g.n, vb, ve, rp_h, ci_h)
+
+    csr = create()
     atos.bfs(csr, sources[0], out=out_h, **knobs)
     csr.close()
-    t_total, e_total = 0.0, 0
-    parts = []
+    steps = args.steps
+    step_s, e_total, parts = [], 0, []
     for k in range(steps):
+        barrier(ws)
         t0 = time.perf_counter()
-        csr = atos.CSR(rp_h, ci_h, device=local)
+        csr = create()
         t1 = time.perf_counter()
         atos.bfs(csr, sources[k % 8], out=out_h, **knobs)
         t2 = time.perf_counter()
         csr.close()
         t3 = time.perf_counter()
-        t_total += t3 - t0
+        step_s.append(allreduce_max(t3 - t0, ws))
         e_total += src_info[k % 8][1]
         parts.append([round(1e3 * (t1 - t0), 1), round(1e3 * (t2 - t1), 1), round(1e3 * (t3 - t2), 1)])
-    per_step = sorted(src_info[k % 8][1] / (sum(parts[k]) / 1e3) / 1e9 for k in range(steps))
-    return {"value": e_total / t_total / 1e9, "unit": "GTEPS", "median_step_value": per_step[steps // 2],
-            "h2d_bytes_per_step": int(rp_h.numel() * 8 + ci_h.numel() * 4),
-            "d2h_bytes_per_step": int(out_h.numel() * 4), "steps": steps, "ms_create_bfs_destroy": parts,
-            "note": "wall clock around host-synchronous C-ABI calls; includes CSR upload + u32 narrowing"}
+    per_step = sorted(src_info[k % 8][1] / step_s[k] / 1e9 for k in range(steps))
+    spread = (max(step_s) - min(step_s)) / float(np.median(step_s))
+    return {"value": e_total / sum(step_s) / 1e9, "unit": "GTEPS", "median_step_value": per_step[steps // 2],
+            "h2d_bytes_per_step": int(allreduce_sum(float(rp_h.numel() * 8 + ci_h.numel() * 4), ws)),
+            "d2h_bytes_per_step": int(allreduce_sum(float(out_h.numel() * 4), ws)), "steps": steps,
+            "step_spread": spread, "ms_create_bfs_destroy": parts,
+            "note": "wall clock around host-synchronous C-ABI calls (max over ranks); includes the CSR upload, "
+                    "u32 narrowing and layout, the BFS, the depth D2H and the destroy"}
 
 
 def cpu_baseline(g, sources, src_info):
@@ -392,7 +484,7 @@ def cpu_baseline(g, sources, src_info):
     d = oracle.bfs(rp, ci, sources[0])
     dt = time.perf_counter() - t0
     edges = int(np.diff(rp)[d != 0xFFFFFFFF].sum())
-    return {"value": edges / dt / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+    return {"value": edges / dt / 1e9, "unit": "GTEPS", "cores": 1, "kind": "oracle", **host_identity(),
             "sample": f"one full serial FIFO BFS (oracle_bfs, gcc -O2) from source {sources[0]} on the same C5 graph",
             "seconds": dt}
 
@@ -593,12 +685,25 @@ def run_apps(args, dev, peak):
         edges.append(st["edges"])
         cols.append(st["colors_used"])
     wm = float(np.mean(wms))
-    alg = GC_BYTES_PER_TASK * np.mean(pops) + GC_BYTES_PER_EDGE * np.mean(edges)
+    # colouring's algorithmic bytes are the MINIMUM work -- one assign and one check task per
+    # vertex (20 B each) and one edge visit per directed edge for each (8 B): 40 n + 16 m.  Overwork (edge
+    # visits beyond the two scans) costs time only; it is reported as edge_visits_per_m next to it.
+    alg = 2 * GC_BYTES_PER_TASK * g.n + 2 * GC_BYTES_PER_EDGE * g.m
+    oracle_counts = {}
+    if not args.no_cpu:
+        import oracle
+        rp, ci = g.numpy()
+        t0 = time.perf_counter()
+        oracle_counts["greedy_id_order"] = oracle.color_greedy(rp, ci)[1]
+        oracle_counts["jones_plassmann_seed1"] = oracle.color_jp(rp, ci, 1)[1]
+        oracle_counts["seconds"] = time.perf_counter() - t0
     res["color"] = {"config": f"C4: Kronecker scale {args.gc_scale} ef 64 seed 4 (n={g.n}, m={g.m}), seed 1, "
                               "CTA worker 1024 / fetch 128 (library default)",
                     "ms_to_converge": float(np.mean(ms)), "ms_min": float(np.min(ms)), "worker_ms": wm,
-                    "colors": int(np.max(cols)), "tasks_per_n": float(np.mean(pops)) / g.n,
-                    "achieved_GBs": alg / (wm / 1e3) / 1e9, "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
+                    "colors": int(np.max(cols)), "oracle_colors": oracle_counts,
+                    "tasks_per_n": float(np.mean(pops)) / g.n,
+                    "algorithmic_bytes": int(alg), "achieved_GBs": alg / (wm / 1e3) / 1e9,
+                    "frac_of_hbm": alg / (wm / 1e3) / 1e9 / peak,
                     "traffic": profile_traffic("color_worker"), "edge_visits_per_m": float(np.mean(edges)) / g.m}
     gpk = micro_peak("random_gather_per_s")
     if gpk:
@@ -677,11 +782,15 @@ def main():
     ap.add_argument("--no-apps", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-bsp", action="store_true", help="skip the bulk-synchronous baselines (atos_*_bsp)")
+    ap.add_argument("--dry-run", action="store_true",
+                    help="CPU/gloo: build this rank's rows and pick the sources, then stop (host-logic test)")
     args = ap.parse_args()
     if args.warmup < 3:
         log("[bench] warmup raised to 3 (timing rules)")
         args.warmup = 3
-    ws, rank, local = dist_setup()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch_under_torchrun(args))
+    ws, rank, local = dist_setup(args)
     if args.impl == "reference":
         run_reference(args, ws, rank)
     else:

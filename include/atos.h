@@ -87,7 +87,8 @@ typedef struct {
                                    of the discrete launches incl. their host round trips), CUDA events */
     uint64_t timeline_len;      /* samples written to cfg->timeline */
     uint64_t flags;             /* bit 0: BFS re-ran with the u32 depth state (depth >= 126 met) */
-    uint64_t reserved[1];
+    uint64_t max_queue_occupancy; /* largest number of published-but-unclaimed items (tail - head) any worker
+                                   saw at a claim (persistent runs; discrete: the largest frontier) */
 } atos_stats;
 
 typedef struct {
@@ -136,7 +137,10 @@ typedef struct {
                                    relaxation (BFS atomicMin on depth, PageRank atomicAdd on residue) and its
                                    activation go straight into the owner's slice and queue; global quiescence
                                    termination; 0 (default) = exchange rounds.  ATOS_ERR_UNSUPPORTED on a
-                                   single-partition or multi-process graph */
+                                   single-partition or multi-process graph, and when persistent=0, dedupe=0,
+                                   worker, fetch_size, queue_capacity, depth_state or engine_variant is set (the
+                                   barrier-free kernel has its own fixed CTA worker); timeout_s is a device
+                                   deadline (the kernel stops itself before the call returns ATOS_ERR_TIMEOUT) */
 } atos_cfg;
 
 /* Fill *cfg with defaults (persistent, app-default worker/fetch, dedupe on). */
@@ -182,6 +186,9 @@ ATOS_API void atos_csr_destroy(atos_csr* g);
 
 /* Query n, m and the number of partitions of a handle (any pointer may be NULL). */
 ATOS_API int atos_csr_info(const atos_csr* g, int64_t* n, int64_t* m, int* num_parts);
+
+/* The layout a handle actually uses (ATOS_LAYOUT_INPUT or ATOS_LAYOUT_DEGREE; AUTO is resolved at creation). */
+ATOS_API int atos_csr_layout(const atos_csr* g, int* layout);
 
 /*
  * Speculative (asynchronous) BFS from `src` (Alg.2): depth_out[v]
@@ -249,6 +256,24 @@ ATOS_API int atos_comm_unique_id(void* id_out, size_t len);
 /* Create the communicator of rank `rank` of `nranks` on CUDA device `device`. Collective. */
 ATOS_API int atos_comm_create(atos_comm** out, int nranks, int rank, const void* id, size_t len, int device);
 ATOS_API void atos_comm_destroy(atos_comm* comm);
+
+/*
+ * Host-staged transport: a communicator whose two exchange steps (per-destination counts, then the
+ * SoA payloads of each round) and termination allreduces go through the
+ * caller's own host collectives instead of NCCL -- e.g. torch.distributed over gloo or MPI.  Used
+ * where NCCL cannot run (several ranks sharing one GPU in tests; no NVLink) and as the reference
+ * transport the NCCL path is checked against.  All buffers are HOST memory owned by the library for
+ * the duration of the call; the callbacks must be collective (every rank calls them in the same
+ * order) and return 0 on success.
+ *   alltoallv: rank r sends send_bytes[p] bytes starting at send + sum(send_bytes[0..p)) to rank p
+ *              and receives recv_bytes[p] bytes from rank p into recv + sum(recv_bytes[0..p)).
+ *   allreduce: in-place sum over ranks of ONE value: dtype 0 = uint64_t, 1 = double.
+ */
+typedef int (*atos_host_alltoallv_fn)(void* user, const void* send, const uint64_t* send_bytes, void* recv,
+                                      const uint64_t* recv_bytes);
+typedef int (*atos_host_allreduce_fn)(void* user, void* value, int dtype);
+ATOS_API int atos_comm_create_host(atos_comm** out, int nranks, int rank, int device,
+                                   atos_host_alltoallv_fn alltoallv, atos_host_allreduce_fn allreduce, void* user);
 
 /*
  * Create this rank's partition of a 1D vertex-block partitioned graph: the

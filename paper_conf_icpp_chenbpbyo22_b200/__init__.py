@@ -62,6 +62,13 @@ class CSR:
         return self
 
     @property
+    def layout(self) -> str:
+        """The layout the library chose at creation: "degree" or "input" (atos_csr_layout)."""
+        v = ctypes.c_int()
+        _lib.check(_lib.load().atos_csr_layout(self.handle, ctypes.byref(v)), "atos_csr_layout")
+        return "degree" if v.value == _lib.LAYOUT_DEGREE else "input"
+
+    @property
     def handle(self):
         if self._h is None:
             raise RuntimeError("CSR handle already closed")
@@ -183,6 +190,48 @@ class Comm:
         _lib.check(lib.atos_comm_create(ctypes.byref(h), nranks, rank, buf, _lib.COMM_ID_BYTES, device),
                    "atos_comm_create")
         self._h, self.nranks, self.rank, self.device = h, nranks, rank, device
+
+    @classmethod
+    def host(cls, nranks: int, rank: int, device: int, group=None) -> "Comm":
+        """Host-staged transport (atos_comm_create_host): the exchange rounds' counts/payload all-to-alls and
+        termination allreduces run over torch.distributed on CPU tensors of `group` (e.g. gloo).  The library
+        still does every step of the path on the GPU; only the bytes between ranks travel through the host."""
+        import torch.distributed as dist
+        lib = _lib.load()
+
+        def a2a(_user, send, send_bytes, recv, recv_bytes):
+            try:
+                sb = [int(send_bytes[i]) for i in range(nranks)]
+                rb = [int(recv_bytes[i]) for i in range(nranks)]
+                src = torch.empty(sum(sb), dtype=torch.uint8)
+                if sum(sb):
+                    ctypes.memmove(src.data_ptr(), send, sum(sb))
+                dst = torch.empty(sum(rb), dtype=torch.uint8)
+                dist.all_to_all_single(dst, src, output_split_sizes=rb, input_split_sizes=sb, group=group)
+                if sum(rb):
+                    ctypes.memmove(recv, dst.data_ptr(), sum(rb))
+                return 0
+            except Exception:  # noqa: BLE001 -- an exception must not cross the C ABI
+                return 1
+
+        def ar(_user, value, dtype):
+            try:
+                ct = ctypes.c_uint64 if dtype == 0 else ctypes.c_double
+                p = ctypes.cast(value, ctypes.POINTER(ct))
+                t = torch.tensor([p[0]], dtype=torch.int64 if dtype == 0 else torch.float64)
+                dist.all_reduce(t, group=group)
+                p[0] = int(t.item()) if dtype == 0 else float(t.item())
+                return 0
+            except Exception:  # noqa: BLE001
+                return 1
+
+        self = cls.__new__(cls)
+        self._cbs = (_lib.HOST_A2A_FN(a2a), _lib.HOST_AR_FN(ar))  # kept alive with the communicator
+        h = ctypes.c_void_p()
+        _lib.check(lib.atos_comm_create_host(ctypes.byref(h), nranks, rank, device, self._cbs[0], self._cbs[1],
+                                             None), "atos_comm_create_host")
+        self._h, self.nranks, self.rank, self.device = h, nranks, rank, device
+        return self
 
     @staticmethod
     def unique_id() -> bytes:

@@ -28,9 +28,14 @@ EXPORTS = [
     "atos_cfg_default", "atos_csr_create", "atos_csr_destroy", "atos_csr_info", "atos_bfs",
     "atos_pagerank", "atos_color", "atos_comm_unique_id", "atos_comm_create", "atos_comm_destroy",
     "atos_csr_create_part", "atos_partition_range", "atos_last_error", "atos_version",
-    "atos_kernel_launches", "atos_bfs_bsp", "atos_pagerank_bsp", "atos_color_bsp", "atos_csr_create_ex",
+    "atos_kernel_launches", "atos_bfs_bsp", "atos_pagerank_bsp", "atos_color_bsp", "atos_csr_create_ex", "atos_csr_layout", "atos_comm_create_host",
 ]
 LAYOUT_AUTO, LAYOUT_INPUT, LAYOUT_DEGREE = 0, 1, 2
+
+# atos_host_alltoallv_fn / atos_host_allreduce_fn (include/atos.h)
+HOST_A2A_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.POINTER(ctypes.c_uint64),
+                               ctypes.c_void_p, ctypes.POINTER(ctypes.c_uint64))
+HOST_AR_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int)
 
 
 class Stats(ctypes.Structure):
@@ -38,11 +43,11 @@ class Stats(ctypes.Structure):
         ("pops", ctypes.c_uint64), ("pushes", ctypes.c_uint64), ("edges", ctypes.c_uint64),
         ("rounds", ctypes.c_uint64), ("bytes_exchanged", ctypes.c_uint64), ("kernel_ms", ctypes.c_double),
         ("residual_sum", ctypes.c_double), ("colors_used", ctypes.c_int64), ("worker_ms", ctypes.c_double),
-        ("timeline_len", ctypes.c_uint64), ("flags", ctypes.c_uint64), ("reserved", ctypes.c_uint64 * 1),
+        ("timeline_len", ctypes.c_uint64), ("flags", ctypes.c_uint64), ("max_queue_occupancy", ctypes.c_uint64),
     ]
 
     def as_dict(self):
-        return {k: getattr(self, k) for k, _ in self._fields_ if k != "reserved"}
+        return {k: getattr(self, k) for k, _ in self._fields_ }
 
 
 class Cfg(ctypes.Structure):
@@ -83,6 +88,7 @@ def load(build_if_missing: bool = True):
             "atos_csr_create_ex": (i32, [ctypes.POINTER(P), i64, i64, P, P, i32, i32, i32, i32]),
             "atos_csr_destroy": (None, [P]),
             "atos_csr_info": (i32, [P, ctypes.POINTER(i64), ctypes.POINTER(i64), ctypes.POINTER(i32)]),
+            "atos_csr_layout": (i32, [P, ctypes.POINTER(i32)]),
             "atos_bfs": (i32, [P, i64, P, ctypes.POINTER(Cfg)]),
             "atos_pagerank": (i32, [P, dbl, dbl, P, ctypes.POINTER(Cfg)]),
             "atos_color": (i32, [P, u64, P, ctypes.POINTER(Cfg)]),
@@ -92,6 +98,7 @@ def load(build_if_missing: bool = True):
             "atos_comm_unique_id": (i32, [P, sz]),
             "atos_comm_create": (i32, [ctypes.POINTER(P), i32, i32, P, sz, i32]),
             "atos_comm_destroy": (None, [P]),
+            "atos_comm_create_host": (i32, [ctypes.POINTER(P), i32, i32, i32, HOST_A2A_FN, HOST_AR_FN, P]),
             "atos_csr_create_part": (i32, [ctypes.POINTER(P), P, i64, i64, i64, i64, P, P, i32]),
             "atos_partition_range": (i32, [i64, i32, i32, ctypes.POINTER(i64), ctypes.POINTER(i64)]),
             "atos_last_error": (ctypes.c_char_p, []),

@@ -112,6 +112,8 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
     return ATOS_ERR_INVALID_ARG;
   }
   r->barrier_free = d.barrier_free;
+  r->knobs_set = (!d.persistent || !d.dedupe || d.worker != 0 || d.fetch_size != 0 || d.queue_capacity != 0 ||
+                  d.depth_state != 0 || d.engine_variant != 0) ? 1 : 0;
   if (r->barrier_free != 0 && r->barrier_free != 1) {
     set_error("barrier_free must be 0 or 1 (got %d)", r->barrier_free);
     return ATOS_ERR_INVALID_ARG;
@@ -284,6 +286,7 @@ int finish_queue(Part& p, cudaStream_t s, atos_stats* st, const char* what) {
     st->pushes += h->stat_pushes.v;
     st->edges += h->stat_edges.v;
     st->timeline_len = h->tl_count.v;
+    if (h->stat_maxocc.v > st->max_queue_occupancy) st->max_queue_occupancy = h->stat_maxocc.v;
   }
   return ATOS_OK;
 }
@@ -462,7 +465,8 @@ void destroy_part(Part& p) {
   p.col = nullptr;
   DevBuf* bufs[] = {&p.ring, &p.ctl, &p.big, &p.bitmap, &p.shadow, &p.vbuf_a, &p.vbuf_b, &p.vbuf_c, &p.scratch,
                     &p.ghost_a, &p.ghost_b, &p.touched, &p.outbox, &p.inbox, &p.out_val, &p.in_val, &p.pack,
-                    &p.bsp_fa, &p.bsp_fb, &p.bsp_off, &p.bsp_tmp, &p.bsp_ctr};
+                    &p.bsp_fa, &p.bsp_fb, &p.bsp_off, &p.bsp_tmp, &p.bsp_ctr, &p.nb_ring, &p.nb_ctl,
+                    &p.nb_peers};
   for (DevBuf* b : bufs) b->release();
   if (p.host_pinned) cudaFreeHost(p.host_pinned);
   p.host_pinned = nullptr;
@@ -630,6 +634,15 @@ int atos_csr_info(const atos_csr* g, int64_t* n, int64_t* m, int* num_parts) {
   if (n) *n = g->n;
   if (m) *m = g->m;
   if (num_parts) *num_parts = g->comm ? g->nranks : g->num_parts;
+  return ATOS_OK;
+}
+
+int atos_csr_layout(const atos_csr* g, int* layout) {
+  if (!g || !layout) {
+    set_error("atos_csr_layout: null argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  *layout = g->relabeled ? ATOS_LAYOUT_DEGREE : ATOS_LAYOUT_INPUT;
   return ATOS_OK;
 }
 

@@ -147,6 +147,7 @@ __global__ void __launch_bounds__(1024) k_color_warp(ColorCtx c, EngineParams P)
     pusher.flush(P.q, P.watchdog_ns);
     wk.complete(P, nready);
   }
+  wk.flush_occ(P);
   flush_stats(P.q, pops, lane_id() == 0 ? edges : 0, lane_id() == 0 ? pusher.total : 0);
 }
 
@@ -309,6 +310,7 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
     pusher.flush(P.q, P.watchdog_ns);
     wk.complete(P, nready);
   }
+  wk.flush_occ(P);
   flush_stats(P.q, pops, edges, lane_id() == 0 ? pusher.total : 0);
 }
 
@@ -387,6 +389,7 @@ __global__ void __launch_bounds__(1024) k_color_thread(ColorCtx c, EngineParams 
     pusher.flush(P.q, P.watchdog_ns);
     wk.complete(P, nready);
   }
+  wk.flush_occ(P);
   flush_stats(P.q, pops, edges, lane == 0 ? pusher.total : 0);
 }
 
@@ -442,6 +445,7 @@ __global__ void k_color_begin(QueueCtl* ctl, unsigned long long n) {
     ctl->stat_pops.v = 0;
     ctl->stat_pushes.v = n;
     ctl->stat_edges.v = 0;
+    ctl->stat_maxocc.v = 0;
     ctl->misc.v = 0;
     ctl->tl_next.v = 0;
     ctl->tl_count.v = 0;

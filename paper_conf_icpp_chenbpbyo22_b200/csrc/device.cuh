@@ -56,6 +56,7 @@ struct QueueCtl {
   Line64 big_rr;      // round-robin slot cursor for big-task registration
   Line64 tl_next;     // timeline: globaltimer of the next sample
   Line64 tl_count;    // timeline: samples taken
+  Line64 stat_maxocc; // largest tail - head a worker saw at a claim (atos_stats.max_queue_occupancy)
 };
 
 struct Ring {

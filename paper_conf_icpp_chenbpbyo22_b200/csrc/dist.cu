@@ -100,7 +100,72 @@ int exchange_loopback(std::vector<ExchangeIO>& io, size_t val_bytes, cudaStream_
   return ATOS_OK;
 }
 
+// Host-staged exchange (atos_comm_create_host): the same two steps as the NCCL path -- per-destination
+// counts, then the SoA payloads -- but through the caller's host alltoallv (e.g. torch.distributed gloo).
+// Each peer's message is [ids: c x u32][values: c x val_bytes].
+static int exchange_host(Comm* c, ExchangeIO& io, size_t val_bytes, cudaStream_t s, uint64_t* bytes_sent) {
+  const int P = c->nranks;
+  std::vector<uint64_t> cb(P, 8), rcnt(P, 0);
+  if (c->h_a2a(c->h_user, io.counts.data(), cb.data(), rcnt.data(), cb.data()) != 0) {
+    set_error("host alltoallv (counts) failed");
+    return ATOS_ERR_NCCL;
+  }
+  uint64_t stot = 0, rtot = 0;
+  for (int p = 0; p < P; ++p) {
+    stot += io.counts[p];
+    rtot += rcnt[p];
+  }
+  const size_t item = 4 + val_bytes;
+  std::vector<char> sbuf(std::max<uint64_t>(stot, 1) * item), rbuf(std::max<uint64_t>(rtot, 1) * item);
+  std::vector<uint32_t> ids(std::max<uint64_t>(stot, 1));
+  std::vector<char> vals(std::max<uint64_t>(stot, 1) * val_bytes);
+  if (stot) {
+    ATOS_CUDA(cudaMemcpyAsync(ids.data(), io.out_vid, stot * 4, cudaMemcpyDeviceToHost, s));
+    ATOS_CUDA(cudaMemcpyAsync(vals.data(), io.out_val, stot * val_bytes, cudaMemcpyDeviceToHost, s));
+  }
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  std::vector<uint64_t> sb(P), rb(P);
+  uint64_t so = 0, b = 0;
+  char* w = sbuf.data();
+  for (int p = 0; p < P; ++p) {
+    const uint64_t k = io.counts[p];
+    memcpy(w, ids.data() + so, k * 4);
+    memcpy(w + k * 4, vals.data() + so * val_bytes, k * val_bytes);
+    w += k * item;
+    so += k;
+    sb[p] = k * item;
+    rb[p] = rcnt[p] * item;
+    if (p != c->rank) b += k * item;
+  }
+  if (c->h_a2a(c->h_user, sbuf.data(), sb.data(), rbuf.data(), rb.data()) != 0) {
+    set_error("host alltoallv (payload) failed");
+    return ATOS_ERR_NCCL;
+  }
+  io.in_total = rtot;
+  ATOS_TRY(io.in_vid->ensure(std::max<uint64_t>(rtot, 1) * 4));
+  ATOS_TRY(io.in_val->ensure(std::max<uint64_t>(rtot, 1) * val_bytes));
+  std::vector<uint32_t> rid(std::max<uint64_t>(rtot, 1));
+  std::vector<char> rval(std::max<uint64_t>(rtot, 1) * val_bytes);
+  const char* q = rbuf.data();
+  uint64_t ro = 0;
+  for (int p = 0; p < P; ++p) {
+    const uint64_t k = rcnt[p];
+    memcpy(rid.data() + ro, q, k * 4);
+    memcpy(rval.data() + ro * val_bytes, q + k * 4, k * val_bytes);
+    q += k * item;
+    ro += k;
+  }
+  if (rtot) {
+    ATOS_CUDA(cudaMemcpyAsync(io.in_vid->p, rid.data(), rtot * 4, cudaMemcpyHostToDevice, s));
+    ATOS_CUDA(cudaMemcpyAsync(io.in_val->p, rval.data(), rtot * val_bytes, cudaMemcpyHostToDevice, s));
+  }
+  ATOS_CUDA(cudaStreamSynchronize(s));  // the host vectors die at return
+  if (bytes_sent) *bytes_sent = b;
+  return ATOS_OK;
+}
+
 int exchange_nccl(Comm* c, ExchangeIO& io, size_t val_bytes, cudaStream_t s, uint64_t* bytes_sent) {
+  if (c->h_a2a) return exchange_host(c, io, val_bytes, s, bytes_sent);
   NcclApi& api = nccl();
   const int P = c->nranks;
   ncclComm_t comm = (ncclComm_t)c->nccl;
@@ -146,6 +211,14 @@ int exchange_nccl(Comm* c, ExchangeIO& io, size_t val_bytes, cudaStream_t s, uin
 }
 
 int allreduce_u64(Comm* c, uint64_t* v, cudaStream_t s) {
+  if (c->h_ar) {
+    ATOS_CUDA(cudaStreamSynchronize(s));
+    if (c->h_ar(c->h_user, v, 0) != 0) {
+      set_error("host allreduce (u64) failed");
+      return ATOS_ERR_NCCL;
+    }
+    return ATOS_OK;
+  }
   static thread_local DevBuf buf;
   ATOS_TRY(buf.ensure(8));
   ATOS_CUDA(cudaMemcpyAsync(buf.p, v, 8, cudaMemcpyHostToDevice, s));
@@ -156,6 +229,14 @@ int allreduce_u64(Comm* c, uint64_t* v, cudaStream_t s) {
 }
 
 int allreduce_f64(Comm* c, double* v, cudaStream_t s) {
+  if (c->h_ar) {
+    ATOS_CUDA(cudaStreamSynchronize(s));
+    if (c->h_ar(c->h_user, v, 1) != 0) {
+      set_error("host allreduce (f64) failed");
+      return ATOS_ERR_NCCL;
+    }
+    return ATOS_OK;
+  }
   static thread_local DevBuf buf;
   ATOS_TRY(buf.ensure(8));
   ATOS_CUDA(cudaMemcpyAsync(buf.p, v, 8, cudaMemcpyHostToDevice, s));
@@ -234,6 +315,29 @@ int atos_comm_create(atos_comm** out, int nranks, int rank, const void* id, size
   c->c.rank = rank;
   c->c.device = device;
   c->c.nccl = comm;
+  *out = c;
+  return ATOS_OK;
+}
+
+int atos_comm_create_host(atos_comm** out, int nranks, int rank, int device, atos_host_alltoallv_fn alltoallv,
+                          atos_host_allreduce_fn allreduce, void* user) {
+  if (!out || nranks < 1 || rank < 0 || rank >= nranks || !alltoallv || !allreduce) {
+    set_error("atos_comm_create_host: invalid argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    cudaGetLastError();
+    set_error("atos_comm_create_host: device %d not available", device);
+    return ATOS_ERR_CUDA;
+  }
+  atos_comm* c = new atos_comm();
+  c->c.nranks = nranks;
+  c->c.rank = rank;
+  c->c.device = device;
+  c->c.h_a2a = alltoallv;
+  c->c.h_ar = allreduce;
+  c->c.h_user = user;
   *out = c;
   return ATOS_OK;
 }

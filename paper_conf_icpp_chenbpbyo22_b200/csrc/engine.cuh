@@ -352,6 +352,7 @@ struct Worker {
   unsigned backoff;
   unsigned long long idle_since;
   unsigned long long deadline;
+  unsigned long long maxocc;  // leader only: largest visible backlog (tail - head) seen at a claim
   ATOS_PH_DECL
 
   __device__ __forceinline__ void init(unsigned char* arena, const EngineParams& P) {
@@ -366,6 +367,7 @@ struct Worker {
     first = true;
     backoff = 32;
     idle_since = 0;
+    maxocc = 0;
     deadline = P.timeout_ns ? globaltimer() + P.timeout_ns : 0;
     if (r == 0) s.ctr[1] = 0;
 #ifdef ATOS_PHASE_PROF
@@ -410,6 +412,7 @@ struct Worker {
           unsigned long long h = ld_relaxed(&q.ctl->head.v);
           const unsigned long long t = ld_relaxed(&q.ctl->tail.v);
           if (h < t) {
+            if (t - h > maxocc) maxocc = t - h;
             const unsigned long long nworkers =
                 (unsigned long long)gridDim.x * (MODE == MODE_CTA ? 1u : (blockDim.x >> 5));
             unsigned long long want = (t - h) / nworkers;
@@ -489,6 +492,11 @@ struct Worker {
       // (compute-sanitizer racecheck: WAR on s.ctr[3] across the loop back-edge)
       group_sync<MODE>();
     }
+  }
+
+  // kernel exit: the leader folds its largest observed backlog into the control block
+  __device__ __forceinline__ void flush_occ(const EngineParams& P) const {
+    if (r == 0 && maxocc) atomicMax(&P.q.ctl->stat_maxocc.v, maxocc);
   }
 
   // All pushes of the batch are published (every warp flushed before this):
@@ -817,6 +825,7 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
     ATOS_PH(PH_COMPLETE);
   }
   ATOS_PH_FLUSH();
+  wk.flush_occ(P);
   flush_stats(q, my_pops, my_edges, lane_id() == 0 ? pusher.total : 0);
 }
 

@@ -65,6 +65,10 @@ struct Part {
 struct Comm {
   int nranks = 1, rank = 0, device = 0;
   void* nccl = nullptr;  // ncclComm_t
+  // host-staged transport (atos_comm_create_host): the caller's collectives move host buffers
+  atos_host_alltoallv_fn h_a2a = nullptr;
+  atos_host_allreduce_fn h_ar = nullptr;
+  void* h_user = nullptr;
 };
 
 // One partition's side of an exchange round.
@@ -118,6 +122,8 @@ struct Resolved {
   int conflict_policy, permute_init, validate, out_where, l2_persist, big_threshold, big_chunk, depth_state;
   int engine_variant;
   int barrier_free;
+  int knobs_set;  // a scheduler knob the barrier-free kernel ignores was set (persistent=0, dedupe=0, worker,
+                  // fetch_size, queue_capacity, depth_state, engine_variant)
   unsigned long long* timeline;
   uint32_t timeline_cap, timeline_interval_ns;
   uint64_t queue_capacity;

@@ -52,7 +52,7 @@ struct NbPeer {  // what a partition exposes to its peers (peer-mapped in a mult
 };
 
 struct NbGlob {
-  unsigned long long abort;  // set by a watchdog
+  unsigned long long abort;  // 1: no-progress watchdog, 2: cfg.timeout_s deadline passed
   unsigned long long edges;  // neighbour-list entries visited
 };
 
@@ -64,6 +64,7 @@ struct NbParams {
   uint32_t S;           // sub-queues per partition (each its own ring + counters; fewer CTAs per head)
   double alpha, eps;
   unsigned long long watchdog_ns;
+  unsigned long long timeout_ns;  // cfg.timeout_s as a device deadline from kernel start (0: none)
 };
 
 __device__ __forceinline__ unsigned long long nb_tag(unsigned long long idx, uint32_t item) {
@@ -142,7 +143,8 @@ __global__ void k_nb_seed(NbParams prm, uint32_t p) {
   }
 }
 
-// The persistent barrier-free worker kernel (one cooperative launch; CTA b serves partition b % P).
+// The persistent barrier-free worker kernel (one cooperative launch; CTA b serves sub-queue b % (P*S), i.e.
+// partition (b % (P*S)) / S).
 // A CTA claims up to kNbBlock items of its partition's ring with ONE CAS (fewer contenders on head than
 // a claim per warp) and expands them as the paper's CTA worker with LBS does.
 template <bool kBfs>
@@ -158,8 +160,12 @@ __global__ void __launch_bounds__(kNbBlock, ATOS_NB_MINB) k_nobarrier(NbParams p
   __shared__ uint32_t s_sq;
   const uint32_t lane = lane_id(), wid = warp_id();
   unsigned long long edges = 0, t_idle = 0, last_done = 0;
+  const unsigned long long t_start = globaltimer();
   while (true) {
     if (threadIdx.x == 0) {
+      // cfg.timeout_s: a device deadline, so the kernel stops on its own (the host never returns while it
+      // still writes the caller's output or the rings)
+      if (prm.timeout_ns && globaltimer() - t_start > prm.timeout_ns) atomicCAS(&prm.glob->abort, 0ull, 2ull);
       uint32_t k = 0, sq = sub0;
       unsigned long long h = 0;
       // own sub-queue first, then the partition's other sub-queues
@@ -368,6 +374,11 @@ static int run_nobarrier(atos_csr* g, bool bfs, double alpha, double eps, double
     set_error("barrier_free: needs a loopback-partitioned graph with 2..%u partitions (got %u)", kNbMaxParts, P);
     return ATOS_ERR_UNSUPPORTED;
   }
+  if (r.knobs_set) {
+    set_error("barrier_free: persistent=0, dedupe=0, worker, fetch_size, queue_capacity, depth_state and "
+              "engine_variant do not apply to the barrier-free kernel (its worker is fixed, DESIGN.md section 7)");
+    return ATOS_ERR_UNSUPPORTED;
+  }
   if (!bfs && r.check_size > 0) {
     set_error("barrier_free: check_size sweeps are single-partition only");
     return ATOS_ERR_UNSUPPORTED;
@@ -382,11 +393,13 @@ static int run_nobarrier(atos_csr* g, bool bfs, double alpha, double eps, double
   std::vector<NbPeer> peers(P);
   for (uint32_t i = 0; i < P; ++i) {
     Part& p = g->parts[i];
-    if (p.v_begin != (int64_t)i * B) {
+    if (p.v_begin != std::min<int64_t>(g->n, (int64_t)i * B)) {  // trailing partitions may be empty
       set_error("barrier_free: partition %u does not start at %u * ceil(n/P)", i, i);
       return ATOS_ERR_INVALID_ARG;
     }
-    const uint64_t cap = nb_pow2((uint64_t)std::max<int64_t>(2 * p.n_local, 1024));
+    // The in-queue bit (BFS) / crossing rule (PageRank) keep at most one entry per vertex outstanding across
+    // a partition's sub-queues, so tail - head <= n_local per ring and n_local slots never lap an unconsumed one.
+    const uint64_t cap = nb_pow2((uint64_t)std::max<int64_t>(p.n_local, 1024));
     ATOS_TRY(p.nb_ring.ensure(S * cap * 8));
     ATOS_TRY(p.nb_ctl.ensure(S * sizeof(NbCtl)));
     ATOS_TRY(p.vbuf_a.ensure((size_t)std::max<int64_t>(p.n_local, 1) * 8));  // PR residue / BFS in-queue bits
@@ -415,7 +428,8 @@ static int run_nobarrier(atos_csr* g, bool bfs, double alpha, double eps, double
     shift = 0;
     while ((1u << shift) < B) ++shift;
   }
-  NbParams prm{(const NbPeer*)base, glob, P, B, shift, S, alpha, eps, r.watchdog_ns};
+  NbParams prm{(const NbPeer*)base, glob, P, B, shift, S, alpha, eps, r.watchdog_ns,
+                r.timeout_s > 0 ? (unsigned long long)(r.timeout_s * 1e9) : 0ull};
   const int gs = 148 * 8;
   if (bfs) {
     const uint32_t o = (uint32_t)(src / B);
@@ -453,11 +467,18 @@ static int run_nobarrier(atos_csr* g, bool bfs, double alpha, double eps, double
     ++g_launches;
   }
   ATOS_CUDA(cudaGetLastError());
-  ATOS_TRY(stream_wait(s, r.timeout_s));
+  if (stream_wait(s, r.timeout_s) == ATOS_ERR_TIMEOUT) {
+    // the device deadline stops the kernel by itself: wait for it before handing the buffers back
+    ATOS_CUDA(cudaStreamSynchronize(s));
+  }
   NbGlob hg{};
   double hsum = 0.0;
   ATOS_CUDA(cudaMemcpy(&hg, glob, sizeof(NbGlob), cudaMemcpyDeviceToHost));
   ATOS_CUDA(cudaMemcpy(&hsum, sum, 8, cudaMemcpyDeviceToHost));
+  if (hg.abort == 2) {
+    set_error("barrier_free %s: timeout_s = %.3f exceeded", bfs ? "BFS" : "PageRank", r.timeout_s);
+    return ATOS_ERR_TIMEOUT;
+  }
   if (hg.abort) {
     set_error("barrier_free %s: no progress for %.1f s (watchdog)", bfs ? "BFS" : "PageRank", r.watchdog_ns * 1e-9);
     return ATOS_ERR_TIMEOUT;

@@ -27,6 +27,7 @@ __device__ __forceinline__ void run_begin(QueueCtl* ctl) {
   ctl->misc.v = 0;
   ctl->tl_next.v = 0;
   ctl->tl_count.v = 0;
+  ctl->stat_maxocc.v = 0;
 }
 
 // Before every persistent launch: over-claims abandoned by a previous kernel
@@ -233,6 +234,7 @@ static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, 
   while (h0 < t0) {
     P.h0 = h0;
     P.t0 = t0;
+    if (st && t0 - h0 > st->max_queue_occupancy) st->max_queue_occupancy = t0 - h0;
     uint64_t grid = (t0 - h0 + items_per_block - 1) / items_per_block;
     if (grid > 0x7FFFFFFFull) grid = 0x7FFFFFFFull;
     void* args[] = {(void*)&app, (void*)&P};

@@ -120,11 +120,16 @@ def permutation(n: int, seed: int, device) -> torch.Tensor:
 
 def rmat(scale: int, edge_factor: int, seed: int, device="cpu", a=0.57, b=0.19, c=0.19,
          permute: bool = True, chunk_pairs: int = 1 << 24, buckets: int | None = None,
-         name: str | None = None) -> Graph:
+         name: str | None = None, rows: tuple[int, int] | None = None) -> Graph:
     """Graph500-initiator RMAT/Kronecker graph, symmetric, no self loops, deduped, ID-permuted.
 
     Pair i, level l: h = hash32(seed, l, i); quadrant (0,0) if h < a*2^32,
     (0,1) if < (a+b)*2^32, (1,0) if < (a+b+c)*2^32, else (1,1); bit (S-1-l).
+
+    rows = (v_begin, v_end): build only those rows (one rank's 1D block, for the multi-process path) --
+    every pair is still drawn, so the rows are bit-identical to the same rows of the full graph; the
+    result's row_ptr has v_end - v_begin + 1 entries (starting at 0) and col holds GLOBAL ids; n stays
+    the global vertex count.
     """
     device = torch.device(device)
     n = 1 << scale
@@ -155,6 +160,9 @@ def rmat(scale: int, edge_factor: int, seed: int, device="cpu", a=0.57, b=0.19, 
         u, w = u[keep], w[keep]
         su = torch.cat([u, w])
         sw = torch.cat([w, u])
+        if rows is not None:
+            mine = (su >= rows[0]) & (su < rows[1])
+            su, sw = su[mine], sw[mine]
         keys = su * n + sw
         if buckets == 1:
             parts[0].append(keys)
@@ -179,8 +187,17 @@ def rmat(scale: int, edge_factor: int, seed: int, device="cpu", a=0.57, b=0.19, 
             del k
     keys = torch.cat(uniq) if uniq else torch.zeros(0, dtype=torch.int64, device=device)
     del uniq
+    nm = name or f"rmat-s{scale}-ef{edge_factor}-seed{seed}"
+    if rows is not None:
+        vb, ve = rows
+        u = keys // n
+        col = (keys - u * n).to(torch.int32)
+        counts = torch.bincount(u - vb, minlength=ve - vb)
+        rp = torch.zeros(ve - vb + 1, dtype=torch.int64, device=device)
+        rp[1:] = torch.cumsum(counts, 0)
+        return Graph(n, int(col.numel()), rp, col, nm + f"-rows{vb}-{ve}")
     rp, col = _csr_from_sorted_keys(keys, n, device)
-    return Graph(n, int(col.numel()), rp, col, name or f"rmat-s{scale}-ef{edge_factor}-seed{seed}")
+    return Graph(n, int(col.numel()), rp, col, nm)
 
 
 def mesh(R: int, C: int, keep_prob: float = 1.0, seed: int = 0, device="cpu",
@@ -235,7 +252,11 @@ def mesh(R: int, C: int, keep_prob: float = 1.0, seed: int = 0, device="cpu",
 
 def pick_source(g: Graph, seed: int) -> int:
     """Seeded choice among non-isolated vertices (DESIGN.md R-BFS-7)."""
-    deg = g.degrees()
+    return pick_source_from_degrees(g.degrees(), seed)
+
+
+def pick_source_from_degrees(deg: torch.Tensor, seed: int) -> int:
+    """pick_source given the (global) degree vector -- e.g. gathered from the ranks' row blocks."""
     cand = torch.nonzero(deg > 0).flatten()
     if cand.numel() == 0:
         return 0

@@ -77,3 +77,28 @@ def test_block_range_matches_library():
         for P in (1, 2, 3, 8):
             for p in range(P):
                 assert dist_host.block_range(n, P, p) == atos.partition_range(n, P, p)
+
+
+def test_bench_dry_run_two_ranks_gloo():
+    """`bench.py --gpus 2 --dry-run` outside torchrun relaunches itself with 2 ranks (gloo here), each rank
+    builds ONLY its row block of the C5-recipe graph (small scale) and picks the 8 sources from the
+    all-gathered degrees: the blocks tile [0, n), their edges add up to the full graph's, and the sources
+    equal the single-process choice."""
+    import json
+    import subprocess
+    import sys
+
+    from paper_conf_icpp_chenbpbyo22_b200 import gen
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--dry-run", "--scale", "12"],
+                       capture_output=True, text=True, timeout=600, cwd=root)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [json.loads(x) for x in r.stdout.splitlines() if x.startswith("{")]
+    assert sorted(x["rank"] for x in lines) == [0, 1]
+    g = gen.rmat(12, 16, 5)
+    lines.sort(key=lambda x: x["rank"])
+    assert lines[0]["v_begin"] == 0 and lines[0]["v_end"] == lines[1]["v_begin"] and lines[1]["v_end"] == g.n
+    assert lines[0]["m_local"] + lines[1]["m_local"] == g.m == lines[0]["m_total"]
+    assert int(g.row_ptr[lines[0]["v_end"]]) == lines[0]["m_local"]
+    want = [gen.pick_source(g, 105 + i) for i in range(8)]
+    assert lines[0]["sources"] == want and lines[1]["sources"] == want

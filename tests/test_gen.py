@@ -98,3 +98,20 @@ def test_config_table():
     g = gen.make_config("C1")
     assert g.n == 65536
     check_csr(g)
+
+
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_rmat_rows_equal_block_of_full_graph(P):
+    """gen.rmat(rows=...) (one rank's 1D block, bench.py --gpus N) == the same rows of the full graph."""
+    from paper_conf_icpp_chenbpbyo22_b200 import dist_host
+    g = gen.rmat(11, 16, 5)
+    for r in range(P):
+        vb, ve = dist_host.block_range(g.n, P, r)
+        part = gen.rmat(11, 16, 5, rows=(vb, ve))
+        rp, ci = dist_host.local_rows(g.row_ptr, g.col, vb, ve)
+        assert part.n == g.n and torch.equal(part.row_ptr, rp) and torch.equal(part.col, ci)
+
+
+def test_pick_source_from_gathered_degrees():
+    g = gen.rmat(10, 8, 2)
+    assert gen.pick_source(g, 105) == gen.pick_source_from_degrees(g.degrees(), 105)

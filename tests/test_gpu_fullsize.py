@@ -8,8 +8,16 @@ that size:
       core) -> every rank within 1e-4 relative, L1 <= 1e-5, one-sided band,
       conservation;
 * C4  Kronecker S20 EF64 colouring: oracle validator (proper, colour <= deg);
-* C5  RMAT S26 BFS (2.1B edges): full oracle BFS from the bench's first source,
-      compared bit for bit, plus the Graph500 validator.
+* C5  RMAT S26 BFS (2.1B edges): full oracle BFS from EVERY one of the 8 sources
+      bench.py times (seeds 105..112), compared bit for bit, plus the Graph500
+      validator;
+* C5  RMAT S26 PageRank (the bench's pagerank_c5 line, degree layout): the
+      residual certificate r = (1-a)1 + a P^T x - x computed by the oracle in one
+      pass; 0 <= r <= eps elementwise implies 0 <= x* - x <= eps x*/(1-a) (the
+      north-star 1e-4 relative / 1e-5 L1 tolerance with 15x / 1.5x margin)
+      without ~185 Jacobi sweeps over 2.1B edges; plus conservation;
+* S23 RMAT PageRank (the first scale where ATOS_LAYOUT_AUTO picks the degree
+      layout): full Jacobi parity like C3.
 Marked slow; they run in the -m gpu suite."""
 import numpy as np
 import pytest
@@ -71,12 +79,63 @@ def test_c4_color_full():
     assert st["colors_used"] == int(c.max().item()) + 1
 
 
-def test_c5_bfs_full():
-    g = gen.make_config("C5", device=DEV)
+def test_s23_pagerank_degree_layout_jacobi():
+    g = gen.rmat(23, 16, 3, device=DEV)
     csr = atos.CSR.from_graph(g)
-    src = gen.pick_source(g, 105)
-    d, st = atos.bfs(csr, src)
+    assert csr.layout == "degree"  # the auto rule's first degree-layout scale (n * 8 B > L2 / 2)
+    r, st = atos.pagerank(csr, 0.85, 1e-6)
     rp, ci = g.numpy()
-    got = as_u32(d)
-    assert oracle.validate_bfs(rp, ci, src, got) == 0
-    np.testing.assert_array_equal(got, oracle.bfs(rp, ci, src))
+    ref, it, ok = oracle.pagerank_jacobi(rp, ci, 0.85)
+    assert ok
+    err = check_pr(rp, ci, r, st, 1e-6, ref=ref)
+    assert abs(err) < 1e-9 * g.n
+
+
+@pytest.fixture(scope="module")
+def c5():
+    g = gen.make_config("C5", device=DEV)
+    rp, ci = g.numpy()
+    sources = [gen.pick_source(g, 105 + i) for i in range(8)]  # the bench's timed sources
+    csr = atos.CSR.from_graph(g)
+    n = g.n
+    del g
+    torch.cuda.empty_cache()
+    yield csr, rp, ci, n, sources
+    csr.close()
+
+
+def test_c5_bfs_full_all_bench_sources(c5):
+    csr, rp, ci, n, sources = c5
+    out = torch.empty(n, dtype=torch.int32, device=DEV)
+    for src in sources:
+        d, st = atos.bfs(csr, src, out=out)
+        got = as_u32(d)
+        assert oracle.validate_bfs(rp, ci, src, got) == 0, src
+        np.testing.assert_array_equal(got, oracle.bfs(rp, ci, src), err_msg=f"source {src}")
+
+
+def test_c5_pagerank_residual_certificate(c5):
+    """C5 PageRank at eps = 1e-6 in the bench's launch configuration (library defaults: degree layout).
+    x* - x = (I - a P^T)^{-1} r with r = (1-a)1 + a P^T x - x (Alg.4's residue), and
+    (I - a P^T)^{-1} >= 0 with (I - a P^T)^{-1} 1 = x*/(1-a).  So
+      -eta <= r <= eps + eta  elementwise   =>   -eta x*/(1-a) <= x* - x <= (eps + eta) x*/(1-a),
+    i.e. every rank within (eps + eta)/(1-a) = 6.7e-6 relative and L1(x/n) <= 6.7e-6 (north star: 1e-4, 1e-5).
+    eta = 1e-12 * max(1, x_w) absorbs the fp64 rounding of the ranks themselves (red.add accumulation)."""
+    csr, rp, ci, n, _ = c5
+    eps, alpha = 1e-6, 0.85
+    assert csr.layout == "degree"
+    r, st = atos.pagerank(csr, alpha, eps)
+    x = r.cpu().numpy() * n  # n = 2^26: exact scaling
+    res = oracle.pagerank_residual(rp, ci, x, alpha)
+    eta = 1e-12 * np.maximum(1.0, x)
+    assert np.all(res >= -eta), f"min residual {res.min()} (rank above the fixed point)"
+    assert np.all(res <= eps + eta), f"max residual {res.max()} > eps"
+    # the certificate's consequences, stated as the north-star tolerances
+    rel_bound = (eps + eta.max()) / (1 - alpha)
+    assert rel_bound < 1e-4
+    assert rel_bound * (x.sum() + res.sum() / (1 - alpha)) / n < 1e-5  # L1(x/n) <= rel_bound * sum(x*)/n
+    # conservation (symmetric graph): sum x + sum r/(1-a) = n - a #isolated, with the library's residues
+    iso = int(np.sum(np.diff(rp) == 0))
+    assert abs(x.sum() + st["residual_sum"] / (1 - alpha) - (n - alpha * iso)) < 1e-9 * n
+    # and the library's residual sum agrees with the certificate's
+    assert abs(st["residual_sum"] - res.sum()) < 1e-6 * n

@@ -190,3 +190,35 @@ def test_bfs_barrier_free_directed_host_output():
     out = torch.empty(7, dtype=torch.int32)
     d, st = atos.bfs(csr, 4, out=out, barrier_free=1)
     np.testing.assert_array_equal(d.numpy().view(np.uint32), oracle.bfs(rp, ci, 4))
+
+
+def test_barrier_free_rejects_ignored_knobs(rmat13):
+    g, rp, ci = rmat13
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=2)
+    for knob in (dict(persistent=0), dict(dedupe=0), dict(worker=32), dict(fetch_size=64),
+                 dict(queue_capacity=1 << 20), dict(depth_state=2), dict(engine_variant=1)):
+        with pytest.raises(RuntimeError, match="UNSUPPORTED"):
+            atos.bfs(csr, 0, barrier_free=1, **knob)
+
+
+def test_barrier_free_trailing_empty_partitions():
+    """n = 9 over P = 8: ceil(9/8) = 2, so parts 5..7 are empty and part 5 starts at min(n, 10) = 9."""
+    rp, ci = G.path(9)
+    csr = csr_of(rp, ci, num_parts=8)
+    for s in (0, 4, 8):
+        d, st = atos.bfs(csr, s, barrier_free=1)
+        np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, s))
+        r, st = atos.pagerank(csr, 0.85, 1e-10, barrier_free=1)
+        check_pr(rp, ci, r, st, 1e-10)
+
+
+def test_barrier_free_device_deadline():
+    """timeout_s is a device deadline: a run longer than it stops itself and the call reports TIMEOUT;
+    the next call on the same handle is unaffected."""
+    g = gen.rmat(16, 16, seed=7)
+    rp, ci = g.numpy()
+    csr = atos.CSR.from_graph(g.to(DEV), num_parts=4)
+    with pytest.raises(RuntimeError, match="TIMEOUT"):
+        atos.pagerank(csr, 0.85, 1e-14, barrier_free=1, timeout_s=1e-5)
+    r, st = atos.pagerank(csr, 0.85, 1e-6, barrier_free=1)
+    check_pr(rp, ci, r, st, 1e-6)
