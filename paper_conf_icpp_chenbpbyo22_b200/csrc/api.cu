@@ -22,24 +22,104 @@ void set_error(const char* fmt, ...) {
   va_end(ap);
 }
 
+namespace {
+struct PoolOf {
+  cudaMemPool_t pool = nullptr;
+  cudaStream_t s = nullptr;  // allocation stream (no kernels run on it)
+};
+std::mutex g_pool_mu;
+PoolOf g_pools[64];
+
+int pool_of(int dev, PoolOf** out) {
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  if (dev < 0 || dev >= 64) {
+    set_error("device %d out of range for the memory pool", dev);
+    return ATOS_ERR_CUDA;
+  }
+  PoolOf& P = g_pools[dev];
+  if (!P.pool) {
+    cudaMemPoolProps props;
+    memset(&props, 0, sizeof(props));
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    ATOS_CUDA(cudaMemPoolCreate(&P.pool, &props));
+    // keep up to 96 GB of freed blocks reserved (a C5 handle plus its workspaces is ~25 GB)
+    uint64_t keep = 96ull << 30;
+    ATOS_CUDA(cudaMemPoolSetAttribute(P.pool, cudaMemPoolAttrReleaseThreshold, &keep));
+    ATOS_CUDA(cudaStreamCreateWithFlags(&P.s, cudaStreamNonBlocking));
+  }
+  *out = &P;
+  return ATOS_OK;
+}
+}  // namespace
+
+int dev_alloc(void** p, size_t bytes) {
+  *p = nullptr;
+  int dev = 0;
+  ATOS_CUDA(cudaGetDevice(&dev));
+  PoolOf* P = nullptr;
+  ATOS_TRY(pool_of(dev, &P));
+  cudaError_t e = cudaMallocFromPoolAsync(p, bytes ? bytes : 16, P->pool, P->s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(P->s);  // usable by every stream from here on
+  if (e != cudaSuccess) {
+    *p = nullptr;
+    cudaGetLastError();
+    set_error("device allocation of %zu bytes failed: %s", bytes, cudaGetErrorString(e));
+    return e == cudaErrorMemoryAllocation ? ATOS_ERR_OOM : ATOS_ERR_CUDA;
+  }
+  return ATOS_OK;
+}
+
+void dev_free(void* p) {
+  if (!p) return;
+  int dev = 0;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) == cudaSuccess) dev = a.device;
+  else cudaGetLastError();
+  PoolOf* P = nullptr;
+  if (pool_of(dev, &P) != ATOS_OK) return;
+  DeviceGuard dg(dev);
+  cudaDeviceSynchronize();  // no kernel may still use the block (cudaFree's own guarantee)
+  cudaFreeAsync(p, P->s);
+  cudaGetLastError();
+}
+
+namespace {
+std::mutex g_pin_mu;
+std::vector<void*> g_pin_free;
+}  // namespace
+
+int pinned_page(void** p) {
+  {
+    std::lock_guard<std::mutex> lk(g_pin_mu);
+    if (!g_pin_free.empty()) {
+      *p = g_pin_free.back();
+      g_pin_free.pop_back();
+      return ATOS_OK;
+    }
+  }
+  ATOS_CUDA(cudaHostAlloc(p, 4096, cudaHostAllocPortable));
+  return ATOS_OK;
+}
+
+void pinned_page_release(void* p) {
+  if (!p) return;
+  std::lock_guard<std::mutex> lk(g_pin_mu);
+  g_pin_free.push_back(p);
+}
+
 int DevBuf::ensure(size_t want) {
   if (want <= bytes && p) return ATOS_OK;
   release();
   if (want == 0) want = 16;
-  cudaError_t e = cudaMalloc(&p, want);
-  if (e != cudaSuccess) {
-    p = nullptr;
-    bytes = 0;
-    cudaGetLastError();
-    set_error("cudaMalloc(%zu) failed: %s", want, cudaGetErrorString(e));
-    return e == cudaErrorMemoryAllocation ? ATOS_ERR_OOM : ATOS_ERR_CUDA;
-  }
+  ATOS_TRY(dev_alloc(&p, want));
   bytes = want;
   return ATOS_OK;
 }
 
 void DevBuf::release() {
-  if (p) cudaFree(p);
+  if (p) dev_free(p);
   p = nullptr;
   bytes = 0;
 }
@@ -170,7 +250,7 @@ int ensure_queue(Part& p, uint64_t cap, cudaStream_t s) {
   }
   if (!p.ctl.p) ATOS_TRY(p.ctl.ensure(sizeof(QueueCtl)));
   if (!p.big.p) ATOS_TRY(p.big.ensure(sizeof(BigTask) * kBigSlots));
-  if (!p.host_pinned) ATOS_CUDA(cudaHostAlloc(&p.host_pinned, 4096, cudaHostAllocDefault));
+  if (!p.host_pinned) ATOS_TRY(pinned_page(&p.host_pinned));
   if (!p.ring_clean) {
     k_ring_init<<<1184, 256, 0, s>>>(p.ring.as<unsigned long long>(), p.ring_cap, p.ctl.as<QueueCtl>(),
                                      p.big.as<BigTask>(), kBigSlots);
@@ -314,67 +394,13 @@ __global__ void k_check_col(const int32_t* col, uint32_t* out, int64_t m, int64_
   }
 }
 
-__global__ void k_max_degree(const uint32_t* row_ptr, int64_t n, unsigned long long* mx) {
-  unsigned long long best = 0;
-  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-    best = max(best, (unsigned long long)(row_ptr[v + 1] - row_ptr[v]));
-  for (int o = 16; o; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
-  if (lane_id() == 0) atomicMax(mx, best);
-}
-
-// Upload rows [v_begin, v_end) of a CSR into part p (device arrays, u32).
-// row_ptr/col are the FULL arrays (host or device); offsets are rebased.
-static int upload_part(Part& p, int64_t n_global, const int64_t* row_ptr, const int32_t* col, int where,
-                       int64_t v_begin, int64_t v_end, int64_t e_begin, int64_t e_end) {
-  p.v_begin = v_begin;
-  p.v_end = v_end;
-  p.n_local = v_end - v_begin;
-  p.m_local = e_end - e_begin;
-  const int64_t nl = p.n_local, ml = p.m_local;
-  ATOS_CUDA(cudaMalloc(&p.row_ptr, (size_t)(nl + 1) * 4));
-  ATOS_CUDA(cudaMalloc(&p.col, (size_t)std::max<int64_t>(ml, 1) * 4));
-  if (where == ATOS_MEM_HOST) {
-    // upload the int64 offsets as they are and narrow on the device (a host loop over n
-    // would cost more than the copy); col goes straight into its final buffer
-    // (whole-graph uploads are also validated there: monotone, 0 .. m -- see validate_host_csr)
-    int64_t* tmp = nullptr;
-    unsigned* bad = nullptr;
-    ATOS_CUDA(cudaMalloc(&tmp, (size_t)(nl + 1) * 8 + 16));
-    bad = (unsigned*)(tmp + nl + 1);
-    ATOS_CUDA(cudaMemset(bad, 0, 4));
-    ATOS_CUDA(cudaMemcpy(tmp, row_ptr + v_begin, (size_t)(nl + 1) * 8, cudaMemcpyHostToDevice));
-    if (v_begin == 0 && v_end == n_global) {
-      k_narrow_row_ptr<<<1024, 256>>>(tmp, p.row_ptr, nl + 1, ml, bad);
-    } else {
-      k_rebase_row_ptr<<<1024, 256>>>(tmp, p.row_ptr, nl + 1, e_begin);
-    }
-    g_launches++;
-    if (ml) ATOS_CUDA(cudaMemcpy(p.col, col + e_begin, (size_t)ml * 4, cudaMemcpyHostToDevice));
-    unsigned hb = 0;
-    ATOS_CUDA(cudaMemcpy(&hb, bad, 4, cudaMemcpyDeviceToHost));
-    cudaFree(tmp);
-    if (hb) {
-      set_error("row_ptr is not non-decreasing (or outside [0, m])");
-      return ATOS_ERR_INVALID_ARG;
-    }
-    return ATOS_OK;
-  }
-  // device input: rebase + narrow on the device
-  k_rebase_row_ptr<<<1024, 256>>>(row_ptr + v_begin, p.row_ptr, nl + 1, e_begin);
-  g_launches++;
-  ATOS_CUDA(cudaGetLastError());
-  if (ml) ATOS_CUDA(cudaMemcpy(p.col, col + e_begin, (size_t)ml * 4, cudaMemcpyDeviceToDevice));
-  ATOS_CUDA(cudaDeviceSynchronize());
-  return ATOS_OK;
-}
-
 // Upload a partition given its LOCAL arrays: row_ptr[0..nl] (any base offset,
 // host or device) and the matching col[0..ml) (global ids).
 int upload_part_local(Part& p, const int64_t* row_ptr, const int32_t* col, int where, int64_t nl, int64_t ml) {
   p.n_local = nl;
   p.m_local = ml;
-  ATOS_CUDA(cudaMalloc(&p.row_ptr, (size_t)(nl + 1) * 4));
-  ATOS_CUDA(cudaMalloc(&p.col, (size_t)std::max<int64_t>(ml, 1) * 4));
+  ATOS_TRY(dev_alloc_t(&p.row_ptr, nl + 1));
+  ATOS_TRY(dev_alloc_t(&p.col, std::max<int64_t>(ml, 1)));
   if (where == ATOS_MEM_HOST) {
     const int64_t base = row_ptr[0];
     std::vector<uint32_t> rp((size_t)nl + 1);
@@ -459,8 +485,8 @@ static int validate_device_csr(int64_t n, int64_t m, const int64_t* row_ptr, con
 }
 
 void destroy_part(Part& p) {
-  if (p.row_ptr) cudaFree(p.row_ptr);
-  if (p.col) cudaFree(p.col);
+  if (p.row_ptr) dev_free(p.row_ptr);
+  if (p.col) dev_free(p.col);
   p.row_ptr = nullptr;
   p.col = nullptr;
   DevBuf* bufs[] = {&p.ring, &p.ctl, &p.big, &p.bitmap, &p.shadow, &p.vbuf_a, &p.vbuf_b, &p.vbuf_c, &p.scratch,
@@ -468,29 +494,8 @@ void destroy_part(Part& p) {
                     &p.bsp_fa, &p.bsp_fb, &p.bsp_off, &p.bsp_tmp, &p.bsp_ctr, &p.nb_ring, &p.nb_ctl,
                     &p.nb_peers};
   for (DevBuf* b : bufs) b->release();
-  if (p.host_pinned) cudaFreeHost(p.host_pinned);
+  pinned_page_release(p.host_pinned);
   p.host_pinned = nullptr;
-}
-
-int compute_max_degree(Part& p, int64_t* out) {
-  unsigned long long* d = nullptr;
-  ATOS_CUDA(cudaMalloc(&d, 8));
-  ATOS_CUDA(cudaMemset(d, 0, 8));
-  if (p.n_local > 0) {
-    k_max_degree<<<512, 256>>>(p.row_ptr, p.n_local, d);
-    g_launches++;
-  }
-  unsigned long long h = 0;
-  ATOS_CUDA(cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost));
-  cudaFree(d);
-  *out = (int64_t)h;
-  return ATOS_OK;
-}
-
-int create_single(atos_csr* g, const int64_t* row_ptr, const int32_t* col, int where) {
-  g->parts.resize(1);
-  ATOS_TRY(upload_part(g->parts[0], g->n, row_ptr, col, where, 0, g->n, 0, g->m));
-  return compute_max_degree(g->parts[0], &g->max_degree);
 }
 
 int create_loopback_parts(atos_csr* g, const int64_t* row_ptr, const int32_t* col, int where);
@@ -584,9 +589,12 @@ int atos_csr_create_ex(atos_csr** out, int64_t n, int64_t m, const int64_t* row_
     return ATOS_ERR_INVALID_ARG;
   }
   DeviceGuard dg(device);
-  if (n > 0) {
-    int rc = where == ATOS_MEM_HOST ? validate_host_csr(n, m, row_ptr, col, num_parts > 1)
-                                    : validate_device_csr(n, m, row_ptr, col);
+  if (n > 0 && where == ATOS_MEM_HOST) {
+    int rc = validate_host_csr(n, m, row_ptr, col, num_parts > 1);  // end points (+ monotone for partitions)
+    if (rc != ATOS_OK) return rc;
+  }
+  if (n > 0 && where == ATOS_MEM_DEVICE && num_parts > 1) {
+    int rc = validate_device_csr(n, m, row_ptr, col);
     if (rc != ATOS_OK) return rc;
   }
   atos_csr* g = new atos_csr();
@@ -594,18 +602,9 @@ int atos_csr_create_ex(atos_csr** out, int64_t n, int64_t m, const int64_t* row_
   g->n = n;
   g->m = m;
   g->num_parts = num_parts;
-  int rc = num_parts == 1 ? create_single(g, row_ptr, col, where) : create_loopback_parts(g, row_ptr, col, where);
-  if (rc == ATOS_OK && where == ATOS_MEM_HOST) rc = validate_uploaded_cols(g);
-  if (rc == ATOS_OK && num_parts == 1 && flags != ATOS_LAYOUT_INPUT) {
-    bool want = flags == ATOS_LAYOUT_DEGREE;
-    if (flags == ATOS_LAYOUT_AUTO) {
-      int l2 = 0;
-      cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, device);
-      const int64_t avg = std::max<int64_t>(1, n > 0 ? m / n : 1);
-      want = n * 8 > (int64_t)l2 / 2 && g->max_degree >= 32 * avg;
-    }
-    if (want) rc = layout_by_degree(g);
-  }
+  // single partition: pipelined upload, validation and layout in one pass (layout.cu); partitions keep the ids
+  int rc = num_parts == 1 ? create_single(g, row_ptr, col, where, flags) : create_loopback_parts(g, row_ptr, col, where);
+  if (rc == ATOS_OK && num_parts > 1 && where == ATOS_MEM_HOST) rc = validate_uploaded_cols(g);
   if (rc != ATOS_OK) {
     atos_csr_destroy(g);
     return rc;

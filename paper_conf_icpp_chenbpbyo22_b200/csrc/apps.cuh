@@ -58,6 +58,7 @@ struct GhostView {
 template <bool PART, bool ACQ = true>
 struct BfsAppT {
   static constexpr bool kAcquirePop = ACQ;
+  static constexpr bool kPfCta = false;  // CTA workers other than the (256,5) build: direct col loads
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
   const uint32_t* __restrict__ row_ptr;
@@ -170,6 +171,7 @@ struct BfsByteAppT {
   // popper's AND is ordered after the pusher's CAS on the same word (the PTX model gives no
   // ordering through the address dependency alone); the AND itself can then stay relaxed.
   static constexpr bool kAcquirePop = true;
+  static constexpr bool kPfCta = false;
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // the 32-bit word holding w's state byte (prefilter and CAS guess)
   const uint32_t* __restrict__ row_ptr;
@@ -274,6 +276,10 @@ struct BfsByteAppT {
 template <bool PART>
 struct PrAppT {
   static constexpr bool kAcquirePop = true;  // atomicExch must follow the pusher's crossing add
+#ifndef ATOS_PF_PR
+#define ATOS_PF_PR 1
+#endif
+  static constexpr bool kPfCta = ATOS_PF_PR != 0 && !PART;  // cp.async col prefetch (C3: 65.3 -> 63.6 ms)
   using Payload = double;  // delta = alpha * rho / deg(v)
   using Token = double;    // residue before our atomicAdd
   const uint32_t* __restrict__ row_ptr;

@@ -324,7 +324,7 @@ int bsp_buffers(Part& p, uint64_t n, bool need_off, BspBufs* b, cudaStream_t s) 
     b->cub_tmp = p.bsp_tmp.p;
     b->cub_bytes = bytes;
   }
-  if (!p.host_pinned) ATOS_CUDA(cudaHostAlloc(&p.host_pinned, 4096, cudaHostAllocDefault));
+  if (!p.host_pinned) ATOS_TRY(pinned_page(&p.host_pinned));
   ATOS_CUDA(cudaMemsetAsync(b->ctr, 0, 64, s));
   return ATOS_OK;
 }

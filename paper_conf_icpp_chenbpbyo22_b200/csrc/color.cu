@@ -16,6 +16,8 @@
 // [base, base+window) are marked; a full window moves to the next one, so
 // colour <= deg(v) always.
 #include <algorithm>
+#include <cstdlib>
+#include <vector>
 
 #include "internal.h"
 
@@ -23,16 +25,30 @@ namespace atos {
 
 constexpr uint32_t kCheck = 0x80000000u;
 constexpr uint32_t kWin = 1024;  // colours per forbidden-set window (warp/CTA workers)
+#ifndef ATOS_GC_DEFER
+#define ATOS_GC_DEFER 1
+#endif
+constexpr bool kDefer = ATOS_GC_DEFER != 0;  // CTA worker: recolour deferral (see k_color_cta)
 #ifndef ATOS_GC_KU
 #define ATOS_GC_KU 4
 #endif
 constexpr int kUc = ATOS_GC_KU;  // CTA worker: edges in flight per thread per expand iteration
+
+// Tools only (build with -DATOS_GC_COUNTS, run with ATOS_GC_COUNTS=<file>): per-vertex counts of
+// assign and check tasks, written as u32 pairs [v][assign, check] to <file> after the run.
+#ifdef ATOS_GC_COUNTS
+static __device__ uint32_t* g_gc_counts;
+#define ATOS_GC_COUNT(v, chk) do { if (g_gc_counts) atomicAdd(g_gc_counts + 2 * (v) + ((chk) ? 1 : 0), 1u); } while (0)
+#else
+#define ATOS_GC_COUNT(v, chk) do {} while (0)
+#endif
 
 struct ColorCtx {
   const uint32_t* __restrict__ row_ptr;
   const uint32_t* __restrict__ col;
   int32_t* color;
   uint32_t* inq;            // assign-task dedupe bitmap (always on for colouring)
+  uint32_t* dfr;            // recolour deferral: bit set while a vertex's last assign was deferred
   unsigned long long seed;
   int literal;              // 1: paper-literal self-recolour policy
   int hash_only;            // 1: conflict priority by hash only (conflict_policy 2)
@@ -55,6 +71,10 @@ struct ColorCtx {
   __device__ __forceinline__ bool claim_assign(uint32_t x) const {
     const uint32_t bit = 1u << (x & 31);
     return !(atom_or_release(inq + (x >> 5), bit) & bit);
+  }
+  // an assign of x is queued and not yet popped (a hint: relaxed read of the dedupe bitmap)
+  __device__ __forceinline__ bool assign_queued(uint32_t x) const {
+    return (ld_relaxed(inq + (x >> 5)) >> (x & 31)) & 1u;
   }
 };
 
@@ -177,12 +197,20 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
     if (!nready) break;
     for (uint32_t k = tid; k < nready; k += B) {
       const uint32_t item = s.item[k], v = item & ~kCheck;
+      ATOS_GC_COUNT(v, item & kCheck);
       const uint32_t st = __ldg(c.row_ptr + v);
       s.start[k] = st;
       s.off[k] = __ldg(c.row_ptr + v + 1) - st;
       flag[k] = 0;
-      if (item & kCheck) cval[k] = ld_relaxed(c.color + v);
-      else atom_and_acquire(c.inq + (v >> 5), ~(1u << (v & 31)));
+      if (item & kCheck) {
+        cval[k] = ld_relaxed(c.color + v);
+      } else {
+        atom_and_acquire(c.inq + (v >> 5), ~(1u << (v & 31)));
+        // recolouring (v already has a colour: it lost a conflict) may defer to higher-priority neighbours,
+        // at most once in a row (flag 3: the previous assign of v was deferred -- colour now)
+        cval[k] = kDefer ? ld_relaxed(c.color + v) : -1;
+        if (kDefer && cval[k] >= 0 && ((ld_relaxed(c.dfr + (v >> 5)) >> (v & 31)) & 1u)) flag[k] = 3;
+      }
     }
     for (uint32_t i = tid; i < nready * 32; i += B) ibm[i] = 0;
     __syncthreads();
@@ -239,6 +267,14 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
         if (!(item & kCheck)) {
           if (cw[k] >= 0 && cw[k] < (int32_t)kWin)
             atomicOr(ibm + own[k] * 32 + (cw[k] >> 5), 1u << (cw[k] & 31));
+          // Recolour deferral: a vertex that lost a conflict does not pick a new colour while a neighbour
+          // that beats it is itself queued for (re)assignment -- both would choose from the same stale
+          // view and collide again (measured: the dense core of C4 was recoloured 8-16x).  It re-queues
+          // itself instead, at most once in a row (unbounded deferral chains rescanned hub rows ~30x
+          // more), so every recolour completes within two pops.
+          if (kDefer && !c.literal && cval[own[k]] >= 0 && !flag[own[k]] && c.assign_queued(w[k]) &&
+              c.loses(item, w[k]))
+            flag[own[k]] = 2;
         } else if (cw[k] == cval[own[k]]) {
           if (c.literal || c.loses(item & ~kCheck, w[k])) flag[own[k]] = 1;
           else if (c.claim_assign(w[k])) { want[k] = true; out[k] = w[k]; }
@@ -254,7 +290,13 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
       uint32_t out = 0;
       if (k < nready) {
         const uint32_t item = s.item[k], v = item & ~kCheck;
-        if (!(item & kCheck)) {
+        if (!(item & kCheck) && flag[k] == 2) {
+          // deferred recolour: back into the queue, colour unchanged
+          if (lane_id() == 0) atomicOr(c.dfr + (v >> 5), 1u << (v & 31));
+          want = lane_id() == 0 && c.claim_assign(v);
+          out = v;
+        } else if (!(item & kCheck)) {
+          if (flag[k] == 3 && lane_id() == 0) atomicAnd(c.dfr + (v >> 5), ~(1u << (v & 31)));
           const uint32_t freebits = ~ibm[k * 32 + lane_id()];
           const unsigned m = __ballot_sync(0xffffffffu, freebits != 0);
           int32_t chosen = -1;
@@ -589,14 +631,16 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   // assign and check tasks of one vertex can both be queued: 2n outstanding + slack
   const uint64_t want = r.queue_capacity ? r.queue_capacity : std::max<uint64_t>(4ull * n, 4096);
   ATOS_TRY(ensure_queue(p, pow2_ceil(want), s));
-  ATOS_TRY(p.bitmap.ensure(((size_t)n + 31) / 32 * 4));
+  const size_t words = ((size_t)n + 31) / 32;
+  ATOS_TRY(p.bitmap.ensure(words * 4 * 2));  // assign dedupe bits, then recolour-deferral bits
   ATOS_TRY(p.scratch.ensure(64));
   Ring q;
   q.slots = p.ring.as<unsigned long long>();
   q.mask = p.ring_cap - 1;
   q.ctl = p.ctl.as<QueueCtl>();
-  ColorCtx c{p.row_ptr, p.col, color, p.bitmap.as<uint32_t>(), seed, r.conflict_policy == 1 ? 1 : 0,
-             r.conflict_policy == 2 ? 1 : 0};
+  ColorCtx c{p.row_ptr, p.col, color, p.bitmap.as<uint32_t>(), p.bitmap.as<uint32_t>() + words, seed,
+             r.conflict_policy == 1 ? 1 : 0, r.conflict_policy == 2 ? 1 : 0};
+  ATOS_CUDA(cudaMemsetAsync(c.dfr, 0, words * 4, s));
   // init: reserve [t, t+n) then publish every vertex
   k_color_begin<<<1, 32, 0, s>>>(q.ctl, n);
   g_launches++;
@@ -625,6 +669,15 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   P.big_chunk = 1;
   const int mode = mode_of(r.worker);
   int rc;
+#ifdef ATOS_GC_COUNTS
+  uint32_t* dcounts = nullptr;
+  const char* gc_out = getenv("ATOS_GC_COUNTS");
+  if (gc_out) {
+    ATOS_CUDA(cudaMalloc(&dcounts, (size_t)n * 8));
+    ATOS_CUDA(cudaMemset(dcounts, 0, (size_t)n * 8));
+  }
+  ATOS_CUDA(cudaMemcpyToSymbol(g_gc_counts, &dcounts, sizeof(dcounts)));
+#endif
   WorkerTimer wt;
   wt.start(s);
   if (mode == MODE_WARP) {
@@ -644,6 +697,20 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
                              (uint64_t)r.fetch * 32 * nw, p, st);
   }
   wt.stop(s);
+#ifdef ATOS_GC_COUNTS
+  if (dcounts) {
+    std::vector<uint32_t> h((size_t)n * 2);
+    cudaDeviceSynchronize();
+    cudaMemcpy(h.data(), dcounts, (size_t)n * 8, cudaMemcpyDeviceToHost);
+    if (FILE* f = fopen(gc_out, "wb")) {
+      fwrite(h.data(), 4, h.size(), f);
+      fclose(f);
+    }
+    cudaFree(dcounts);
+    dcounts = nullptr;
+    cudaMemcpyToSymbol(g_gc_counts, &dcounts, sizeof(dcounts));
+  }
+#endif
   if (rc != ATOS_OK) return rc;
   if (st) st->worker_ms += wt.elapsed();
   rc = finish_queue(p, s, st, "color");

@@ -148,6 +148,22 @@ __device__ __forceinline__ void tl_sample(const EngineParams& P) {
 
 constexpr uint32_t kGoBig = 0xFFFFFFFFu;
 
+// ---------------------------------------------------------- col prefetch (cp.async)
+// PF (kernel template flag): the CTA worker's expand loop stages the NEXT iteration's neighbour ids into a
+// per-warp shared-memory double buffer with cp.async (no registers held across the iteration), so the col
+// load's latency overlaps the current iteration's state gathers and atomics instead of adding to them.
+// Measured (tools/ab.py, profiles/r02_ab_*): mesh / road-like BFS and PageRank faster, scale-free BFS
+// slower (its hub spans are already one coalesced load per lane) -- the launcher picks it per graph.
+constexpr uint32_t kPfKU = 4;                              // buffer sized for up to 4 edges per lane
+constexpr uint32_t kPfWarpBytes = 2u * 32u * kPfKU * 6u;   // 2 stages x (u32 id + u16 owner) per edge slot
+__device__ __forceinline__ void cp_async4(void* smem, const void* gmem, unsigned long long pol) {
+  const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(sa), "l"(gmem), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+
 template <class Payload>
 __device__ __forceinline__ unsigned long long payload_bits(const Payload& p) {
   static_assert(sizeof(Payload) <= 8, "payload must fit 8 bytes");
@@ -532,7 +548,7 @@ __device__ __forceinline__ void flush_stats(const Ring& q, unsigned long long po
 #ifndef ATOS_MAXT
 #define ATOS_MAXT 1024
 #endif
-template <class App, int MODE, bool PERSIST, int KU = kU, int MINB = ATOS_MINB>
+template <class App, int MODE, bool PERSIST, int KU = kU, int MINB = ATOS_MINB, bool PF = false>
 __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_worker(App app, EngineParams P) {
   using Payload = typename App::Payload;
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -676,6 +692,92 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
       ph_exp0 = ph_last;
       ph_total = total;
 #endif
+      if constexpr (PF) {
+        // per-warp double buffer after the owner table: [stage][KU*32] u32 ids, then [stage][KU*32] u16 owners
+        uint32_t* pf_id = (uint32_t*)((unsigned char*)(cown + kCown) + (size_t)warp_id() * kPfWarpBytes);
+        uint16_t* pf_own = (uint16_t*)(pf_id + 2 * 32 * kPfKU);
+        const uint32_t step = G * KU;
+        // stage: the owners of this warp's span of iteration `base` and cp.async of its neighbour ids
+        auto stage = [&](uint32_t base, uint32_t buf) {
+          const uint32_t wfirst = base + (r & ~31u) * KU;
+          uint16_t* ob_ = pf_own + buf * 32 * kPfKU;
+          uint32_t* ib_ = pf_id + buf * 32 * kPfKU;
+          if (wfirst >= total) {
+#pragma unroll
+            for (int k = 0; k < KU; ++k) ob_[k * 32 + lane_id()] = 0xFFFFu;
+            return;
+          }
+          const uint32_t wlast = min(wfirst + wspan, total) - 1;
+          uint32_t ob = 0;
+          if (table) {
+            const uint32_t c = wfirst / wspan;
+            ob = lane_id() == 0 ? cown[c] : (c + 1 < nchunk ? cown[c + 1] : nready - 1);
+          } else if (lane_id() < 2) {
+            const uint32_t e = lane_id() == 0 ? wfirst : wlast;
+            uint32_t l = 0, h = nready;
+            while (h - l > 1) {
+              const uint32_t mid = (l + h) >> 1;
+              if (s.off[mid] <= e) l = mid; else h = mid;
+            }
+            ob = l;
+          }
+          const uint32_t olo = __shfl_sync(0xffffffffu, ob, 0), ohi = __shfl_sync(0xffffffffu, ob, 1);
+          // lane-strided edges e = wfirst + k*32 + lane: every cp.async instruction covers 32 consecutive
+          // flattened edges; owners by binary search over [olo, ohi], monotone in k
+          uint32_t o = olo;
+#pragma unroll
+          for (int k = 0; k < KU; ++k) {
+            const uint32_t e = wfirst + k * 32 + lane_id();
+            uint16_t own = 0xFFFFu;
+            if (e <= wlast) {
+              uint32_t l = o, h = ohi + 1;
+              while (h - l > 1) {
+                const uint32_t mid = (l + h) >> 1;
+                if (s.off[mid] <= e) l = mid; else h = mid;
+              }
+              o = l;
+              own = (uint16_t)l;
+              cp_async4(ib_ + k * 32 + lane_id(), app.col + s.start[l] + (e - s.off[l]), app.pol_first);
+              ATOS_DBG_EDGE(P, s.start[l] + (e - s.off[l]));
+            }
+            ob_[k * 32 + lane_id()] = own;
+          }
+        };
+        stage(0, 0);
+        cp_async_commit();
+        uint32_t buf = 0;
+        for (uint32_t base = 0; base < total; base += step, buf ^= 1u) {
+          stage(base + step, buf ^ 1u);
+          cp_async_commit();
+          cp_async_wait1();  // this iteration's group has landed
+          __syncwarp();
+          const uint32_t wfirst = base + (r & ~31u) * KU;
+          if (wfirst >= total) continue;  // warp-uniform
+          const uint16_t* ob_ = pf_own + buf * 32 * kPfKU;
+          const uint32_t* ib_ = pf_id + buf * 32 * kPfKU;
+          uint32_t w[KU], own[KU];
+          typename App::Token tk[KU];
+          bool want[KU];
+          uint32_t out[KU];
+#pragma unroll
+          for (int k = 0; k < KU; ++k) {
+            own[k] = ob_[k * 32 + lane_id()];
+            if (own[k] != 0xFFFFu) w[k] = ib_[k * 32 + lane_id()];
+          }
+#pragma unroll
+          for (int k = 0; k < KU; ++k)
+            if (own[k] != 0xFFFFu) tk[k] = app.pre(s.pay[own[k]], w[k]);
+#pragma unroll
+          for (int k = 0; k < KU; ++k) {
+            want[k] = false;
+            out[k] = 0;
+            if (own[k] != 0xFFFFu) want[k] = app.post(s.pay[own[k]], w[k], tk[k], out[k]);
+          }
+          pusher.push_n<KU>(q, want, out, P.watchdog_ns);
+        }
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        __syncwarp();
+      } else {
       for (uint32_t base = 0; base < total; base += G * KU) {
         const uint32_t wfirst = base + (r & ~31u) * KU;
         if (wfirst >= total) continue;  // warp-uniform; no collective below is skipped by part of a warp
@@ -722,6 +824,30 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
           pusher.push_n<KU>(q, want, out, P.watchdog_ns);
           continue;
         }
+        uint32_t own[KU];
+        bool val[KU];
+#ifdef ATOS_LBS_STRIDED
+        // lane-strided: edge wfirst + k*32 + lane (each col load instruction covers 32 consecutive
+        // flattened edges); owners by binary search over [olo, ohi], monotone in k
+        uint32_t o = olo;
+#pragma unroll
+        for (int k = 0; k < KU; ++k) {
+          const uint32_t e = wfirst + k * 32 + lane_id();
+          val[k] = e <= wlast;
+          if (val[k]) {
+            uint32_t l = o, h = ohi + 1;
+            while (h - l > 1) {
+              const uint32_t mid = (l + h) >> 1;
+              if (s.off[mid] <= e) l = mid; else h = mid;
+            }
+            o = l;
+            own[k] = l;
+            const uint32_t ce = s.start[l] + (e - s.off[l]);
+            w[k] = app.neighbor(ce);
+            ATOS_DBG_EDGE(P, ce);
+          }
+        }
+#else
         const uint32_t e0 = wfirst + lane_id() * KU;
         uint32_t o = olo;
         {
@@ -732,8 +858,6 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
           }
           o = l;
         }
-        uint32_t own[KU];
-        bool val[KU];
 #pragma unroll
         for (int k = 0; k < KU; ++k) {
           const uint32_t e = e0 + k;
@@ -746,6 +870,7 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
             ATOS_DBG_EDGE(P, ce);
           }
         }
+#endif
 #pragma unroll
         for (int k = 0; k < KU; ++k)
           if (val[k]) tk[k] = app.pre(s.pay[own[k]], w[k]);
@@ -757,6 +882,7 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
         }
         pusher.push_n<KU>(q, want, out, P.watchdog_ns);
       }
+      }  // !PF
     } else if (MODE == MODE_WARP) {
       for (uint32_t k = 0; k < nready; ++k) {
         const uint32_t st = s.start[k], dg = s.off[k];
@@ -831,11 +957,12 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
 
 // Host-side helper: dynamic shared memory for a launch.
 template <class Payload>
-inline size_t relax_worker_smem(int mode, uint32_t block, uint32_t fetch) {
+inline size_t relax_worker_smem(int mode, uint32_t block, uint32_t fetch, bool pf = false) {
   uint32_t nwarps = block / 32;
   uint32_t K = mode == MODE_THREAD ? 32u * fetch : fetch;
   uint32_t groups = mode == MODE_CTA ? 1u : nwarps;
-  return (size_t)nwarps * kPushBuf * 4 + group_smem_bytes<Payload>(K) * groups + (mode == MODE_CTA ? kCown * 4 : 0);
+  return (size_t)nwarps * kPushBuf * 4 + group_smem_bytes<Payload>(K) * groups +
+         (mode == MODE_CTA ? kCown * 4 + (pf ? (size_t)nwarps * kPfWarpBytes : 0) : 0);
 }
 
 }  // namespace atos

@@ -34,6 +34,19 @@ extern std::atomic<uint64_t> g_launches;
     if (rc_ != ATOS_OK) return rc_; \
   } while (0)
 
+// Device memory of the library: a stream-ordered pool per device (cudaMallocFromPoolAsync) whose release
+// threshold keeps freed blocks reserved, so the graph arrays and workspaces of a handle created and
+// destroyed per step (the e2e path) are re-used instead of being mapped and unmapped by cudaMalloc /
+// cudaFree every time.  dev_free waits for the device first (the same guarantee cudaFree gives).
+int dev_alloc(void** p, size_t bytes);
+void dev_free(void* p);
+// 4 KB pinned host pages (control-block reads), recycled through a free list: no cudaHostAlloc /
+// cudaFreeHost per handle
+int pinned_page(void** p);
+void pinned_page_release(void* p);
+template <class T>
+inline int dev_alloc_t(T** p, size_t count) { return dev_alloc((void**)p, count * sizeof(T)); }
+
 // a device allocation owned by the handle
 struct DevBuf {
   void* p = nullptr;
@@ -198,7 +211,7 @@ struct WorkerTimer {
 int stream_wait(cudaStream_t s, double timeout_s);
 
 // degree layout (layout.cu)
-int layout_by_degree(atos_csr* g);
+int create_single(atos_csr* g, const int64_t* row_ptr, const int32_t* col, int where, int flags);
 template <class T>
 int layout_scatter(const atos_csr* g, const T* in, T* out, cudaStream_t s);
 int64_t layout_vertex(const atos_csr* g, int64_t v);  // caller id -> internal id (-1 on a CUDA error)

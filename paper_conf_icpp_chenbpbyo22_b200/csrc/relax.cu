@@ -187,24 +187,29 @@ __global__ void k_pr_sweep(const double* res, int64_t n, double eps, Ring q, uin
 }
 
 // -------------------------------------------------------------- launchers
+#ifndef ATOS_PF_LOWDEG
+#define ATOS_PF_LOWDEG 1
+#endif
+constexpr bool kPfLowDegree = ATOS_PF_LOWDEG != 0;
+
 static inline uint64_t pow2_at_least(uint64_t x) {
   uint64_t c = 1;
   while (c < x) c <<= 1;
   return c;
 }
 
-template <class App, int MODE, int KU = kU, int MINB = ATOS_MINB>
+template <class App, int MODE, int KU = kU, int MINB = ATOS_MINB, bool PF = false>
 static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, int block,
                              Part& p, atos_stats* st) {
   using Payload = typename App::Payload;
   cudaStream_t s = r.stream;
-  const size_t smem = relax_worker_smem<Payload>(MODE, block, P.fetch);
+  const size_t smem = relax_worker_smem<Payload>(MODE, block, P.fetch, PF && MODE == MODE_CTA);
   if (smem > 227 * 1024) {
     set_error("fetch_size %d with worker %d needs %zu B of shared memory (> 227 KB)", r.fetch, r.worker, smem);
     return ATOS_ERR_INVALID_ARG;
   }
   if (r.persistent) {
-    const void* fn = (const void*)k_relax_worker<App, MODE, true, KU, MINB>;
+    const void* fn = (const void*)k_relax_worker<App, MODE, true, KU, MINB, PF>;
     if (smem > 48 * 1024) ATOS_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int grid = 0;
     ATOS_TRY(persistent_grid(fn, block, smem, &grid));
@@ -219,7 +224,7 @@ static int launch_relax_mode(const App& app, EngineParams P, const Resolved& r, 
   }
   // discrete: one launch per frontier [h0, t0); the host reads the
   // tail after each launch -- the per-frontier host round trip the paper measures.
-  const void* fn = (const void*)k_relax_worker<App, MODE, false, KU, MINB>;
+  const void* fn = (const void*)k_relax_worker<App, MODE, false, KU, MINB, PF>;
   if (smem > 48 * 1024) ATOS_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const uint64_t K = MODE == MODE_THREAD ? 32ull * P.fetch : P.fetch;
   const uint64_t groups_per_block = MODE == MODE_CTA ? 1 : block / 32;
@@ -317,11 +322,16 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
     // 256-thread CTA workers: the (256, 5) register budget (48 regs, 40 warps per SM); kU = 2 edges
     // in flight per thread on low-degree graphs (meshes / road-like: m/n < 8), 4 otherwise.  Measured
     // (tools/sweep.py, one B200): C5 BFS 15.25 -> 14.8 ms, C2 mesh 58 -> 47 ms, road 68 -> 52 ms.
+    // Low-degree graphs also stage the next iteration's col loads with cp.async (PF): their LBS spans cross
+    // many short rows, so the col load is a full extra round trip per iteration (mesh 48.5 -> 46.8 ms, road
+    // 55 -> 49.6 ms); scale-free BFS keeps the direct loads (13.4 -> 15.9 ms with PF).
     if (block == 256 && r.persistent && r.engine_variant != 1) {
       const bool low_degree = p.n_local > 0 && p.m_local < 8 * p.n_local;
-      if (low_degree) return launch_relax_mode<App, MODE_CTA, 2, 5>(app, P, r, block, p, st);
+      if (low_degree) return launch_relax_mode<App, MODE_CTA, 2, 5, kPfLowDegree>(app, P, r, block, p, st);
       return launch_relax_mode<App, MODE_CTA, 4, 5>(app, P, r, block, p, st);
     }
+    if (App::kPfCta && r.persistent && r.engine_variant != 1)
+      return launch_relax_mode<App, MODE_CTA, kU, ATOS_MINB, true>(app, P, r, block, p, st);
     return launch_relax_mode<App, MODE_CTA>(app, P, r, block, p, st);
   }
   if (mode == MODE_WARP) return launch_relax_mode<App, MODE_WARP>(app, P, r, block, p, st);

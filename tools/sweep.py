@@ -35,6 +35,7 @@ def main():
     ap.add_argument("--grid", default=None)
     ap.add_argument("--extra", default="", help="k=v,k=v knobs added to every configuration")
     ap.add_argument("--layout", default="auto", help="CSR layout: auto | degree | input")
+    ap.add_argument("--sources", type=int, default=1, help="bfs-rmat: cycle over the bench's first N sources")
     a = ap.parse_args()
     extra = {k: int(v) for k, v in (kv.split("=") for kv in a.extra.split(",") if kv)}
     if a.app in ("bfs-mesh", "bfs-road"):
@@ -42,7 +43,8 @@ def main():
         src = gen.mesh_centre_source(g, a.side, a.side)
     elif a.app == "bfs-rmat":
         g = gen.rmat(a.scale or 26, 16, 5, device="cuda")
-        src = gen.pick_source(g, 105)
+        srcs = [gen.pick_source(g, 105 + i) for i in range(a.sources)]
+        src = srcs[0]
     elif a.app == "pr":
         g = gen.rmat(a.scale or 22, 16, 3, device="cuda")
         src = None
@@ -60,8 +62,10 @@ def main():
         knobs = dict(worker=w, fetch_size=f, persistent=p, timeout_s=20, **extra)
         ms, wms, st = [], [], None
         try:
-            for _ in range(a.reps + 1):
-                if a.app.startswith("bfs"):
+            for it in range(a.reps + 1):
+                if a.app == "bfs-rmat":
+                    _, st = atos.bfs(csr, srcs[it % len(srcs)], **knobs)
+                elif a.app.startswith("bfs"):
                     _, st = atos.bfs(csr, src, **knobs)
                 elif a.app == "pr":
                     _, st = atos.pagerank(csr, 0.85, 1e-6, **knobs)
