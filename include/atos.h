@@ -141,6 +141,11 @@ typedef struct {
                                    worker, fetch_size, queue_capacity, depth_state or engine_variant is set (the
                                    barrier-free kernel has its own fixed CTA worker); timeout_s is a device
                                    deadline (the kernel stops itself before the call returns ATOS_ERR_TIMEOUT) */
+    int      recolor_spread;    /* colouring, CTA worker: 0/1 (default) = every assign takes the smallest free
+                                   colour (Alg.6 find_min_color); k > 1 = the a-th RECOLOUR of a
+                                   vertex takes the j-th smallest free colour <= deg(v), j = hash mod
+                                   min(2^(a-1), k) -- breaks repeated collisions in dense cores at the price
+                                   of more colours (DESIGN.md R-GC-10) */
 } atos_cfg;
 
 /* Fill *cfg with defaults (persistent, app-default worker/fetch, dedupe on). */
@@ -285,6 +290,17 @@ ATOS_API int atos_comm_create_host(atos_comm** out, int nranks, int rank, int de
 ATOS_API int atos_csr_create_part(atos_csr** out, atos_comm* comm, int64_t n_global, int64_t v_begin,
                          int64_t v_end, int64_t m_local, const int64_t* row_ptr_local,
                          const int32_t* col_global, int where);
+
+/*
+ * Gather the ranks' output slices (atos_bfs depth / atos_pagerank rank, device pointers on each rank's
+ * device, slice [v_begin, v_end) of atos_partition_range) into ONE array of n_global elements of
+ * elem_bytes each on rank 0: out_root is a device pointer on rank 0's device (ignored elsewhere).
+ * Collective over the communicator (NCCL point-to-point, or the host transport of
+ * atos_comm_create_host); enqueued on `stream` (cudaStream_t, NULL = default) and complete on return.
+ * This is the multi-process form of SURVEY 8(b)'s "outputs on the first device".
+ */
+ATOS_API int atos_comm_gather(atos_comm* comm, int64_t n_global, const void* slice, size_t elem_bytes,
+                              void* out_root, void* stream);
 
 /* Block partition used by the library: rank r owns [r*ceil(n/P), min(n,(r+1)*ceil(n/P))). */
 ATOS_API int atos_partition_range(int64_t n, int nparts, int part, int64_t* v_begin, int64_t* v_end);

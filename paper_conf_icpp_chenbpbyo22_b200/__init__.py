@@ -254,6 +254,17 @@ class Comm:
         g._comm_ref = self
         return g
 
+    def gather(self, n_global: int, slice_: torch.Tensor, out: torch.Tensor | None = None):
+        """atos_comm_gather: every rank's output slice -> one n_global array on rank 0 (None elsewhere)."""
+        lib = _lib.load()
+        if self.rank == 0 and out is None:
+            out = torch.empty(n_global, dtype=slice_.dtype, device=slice_.device)
+        stream = torch.cuda.current_stream(slice_.device)
+        _lib.check(lib.atos_comm_gather(self._h, n_global, _ptr(slice_), slice_.element_size(),
+                                        _ptr(out) if out is not None else None, ctypes.c_void_p(stream.cuda_stream)),
+                   "atos_comm_gather")
+        return out
+
     def close(self):
         if getattr(self, "_h", None) is not None:
             _lib.load().atos_comm_destroy(self._h)

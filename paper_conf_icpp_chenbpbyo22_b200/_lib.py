@@ -28,7 +28,7 @@ EXPORTS = [
     "atos_cfg_default", "atos_csr_create", "atos_csr_destroy", "atos_csr_info", "atos_bfs",
     "atos_pagerank", "atos_color", "atos_comm_unique_id", "atos_comm_create", "atos_comm_destroy",
     "atos_csr_create_part", "atos_partition_range", "atos_last_error", "atos_version",
-    "atos_kernel_launches", "atos_bfs_bsp", "atos_pagerank_bsp", "atos_color_bsp", "atos_csr_create_ex", "atos_csr_layout", "atos_comm_create_host",
+    "atos_kernel_launches", "atos_bfs_bsp", "atos_pagerank_bsp", "atos_color_bsp", "atos_csr_create_ex", "atos_csr_layout", "atos_comm_create_host", "atos_comm_gather",
 ]
 LAYOUT_AUTO, LAYOUT_INPUT, LAYOUT_DEGREE = 0, 1, 2
 
@@ -60,7 +60,7 @@ class Cfg(ctypes.Structure):
         ("stats", ctypes.POINTER(Stats)), ("l2_persist", ctypes.c_int), ("big_threshold", ctypes.c_int),
         ("big_chunk", ctypes.c_int), ("timeline_cap", ctypes.c_uint32), ("timeline", ctypes.c_void_p),
         ("timeline_interval_ns", ctypes.c_uint32), ("depth_state", ctypes.c_int), ("engine_variant", ctypes.c_int),
-        ("barrier_free", ctypes.c_int),
+        ("barrier_free", ctypes.c_int), ("recolor_spread", ctypes.c_int),
     ]
 
 
@@ -98,6 +98,7 @@ def load(build_if_missing: bool = True):
             "atos_comm_unique_id": (i32, [P, sz]),
             "atos_comm_create": (i32, [ctypes.POINTER(P), i32, i32, P, sz, i32]),
             "atos_comm_destroy": (None, [P]),
+            "atos_comm_gather": (i32, [P, i64, P, sz, P, P]),
             "atos_comm_create_host": (i32, [ctypes.POINTER(P), i32, i32, i32, HOST_A2A_FN, HOST_AR_FN, P]),
             "atos_csr_create_part": (i32, [ctypes.POINTER(P), P, i64, i64, i64, i64, P, P, i32]),
             "atos_partition_range": (i32, [i64, i32, i32, ctypes.POINTER(i64), ctypes.POINTER(i64)]),

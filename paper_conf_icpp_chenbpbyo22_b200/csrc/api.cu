@@ -192,6 +192,11 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
     return ATOS_ERR_INVALID_ARG;
   }
   r->barrier_free = d.barrier_free;
+  r->recolor_spread = d.recolor_spread;
+  if (r->recolor_spread < 0 || r->recolor_spread > 64) {
+    set_error("recolor_spread must be in [0, 64] (got %d)", r->recolor_spread);
+    return ATOS_ERR_INVALID_ARG;
+  }
   r->knobs_set = (!d.persistent || !d.dedupe || d.worker != 0 || d.fetch_size != 0 || d.queue_capacity != 0 ||
                   d.depth_state != 0 || d.engine_variant != 0) ? 1 : 0;
   if (r->barrier_free != 0 && r->barrier_free != 1) {

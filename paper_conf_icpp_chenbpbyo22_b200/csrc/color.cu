@@ -25,10 +25,7 @@ namespace atos {
 
 constexpr uint32_t kCheck = 0x80000000u;
 constexpr uint32_t kWin = 1024;  // colours per forbidden-set window (warp/CTA workers)
-#ifndef ATOS_GC_DEFER
-#define ATOS_GC_DEFER 1
-#endif
-constexpr bool kDefer = ATOS_GC_DEFER != 0;  // CTA worker: recolour deferral (see k_color_cta)
+
 #ifndef ATOS_GC_KU
 #define ATOS_GC_KU 4
 #endif
@@ -48,7 +45,8 @@ struct ColorCtx {
   const uint32_t* __restrict__ col;
   int32_t* color;
   uint32_t* inq;            // assign-task dedupe bitmap (always on for colouring)
-  uint32_t* dfr;            // recolour deferral: bit set while a vertex's last assign was deferred
+  uint8_t* att;             // recolours per vertex so far (saturating; a heuristic, races are harmless)
+  uint32_t spread;          // cfg.recolor_spread (CTA worker): 1 = Alg.6's smallest free colour on every assign
   unsigned long long seed;
   int literal;              // 1: paper-literal self-recolour policy
   int hash_only;            // 1: conflict priority by hash only (conflict_policy 2)
@@ -72,10 +70,7 @@ struct ColorCtx {
     const uint32_t bit = 1u << (x & 31);
     return !(atom_or_release(inq + (x >> 5), bit) & bit);
   }
-  // an assign of x is queued and not yet popped (a hint: relaxed read of the dedupe bitmap)
-  __device__ __forceinline__ bool assign_queued(uint32_t x) const {
-    return (ld_relaxed(inq + (x >> 5)) >> (x & 31)) & 1u;
-  }
+
 };
 
 // ---------------------------------------------------------------- warp worker
@@ -206,10 +201,14 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
         cval[k] = ld_relaxed(c.color + v);
       } else {
         atom_and_acquire(c.inq + (v >> 5), ~(1u << (v & 31)));
-        // recolouring (v already has a colour: it lost a conflict) may defer to higher-priority neighbours,
-        // at most once in a row (flag 3: the previous assign of v was deferred -- colour now)
-        cval[k] = kDefer ? ld_relaxed(c.color + v) : -1;
-        if (kDefer && cval[k] >= 0 && ((ld_relaxed(c.dfr + (v >> 5)) >> (v & 31)) & 1u)) flag[k] = 3;
+        // a recolour (v already holds a colour: it lost a conflict) may spread its choice (see finalize):
+        // flag[k] = the spread for this attempt, doubling with every recolour of v
+        cval[k] = c.spread > 1 ? ld_relaxed(c.color + v) : -1;
+        if (cval[k] >= 0 && !c.literal) {
+          const uint32_t a = c.att[v];
+          flag[k] = min(1u << min(a, 15u), c.spread);
+          c.att[v] = (uint8_t)min(a + 1, 15u);
+        }
       }
     }
     for (uint32_t i = tid; i < nready * 32; i += B) ibm[i] = 0;
@@ -267,14 +266,6 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
         if (!(item & kCheck)) {
           if (cw[k] >= 0 && cw[k] < (int32_t)kWin)
             atomicOr(ibm + own[k] * 32 + (cw[k] >> 5), 1u << (cw[k] & 31));
-          // Recolour deferral: a vertex that lost a conflict does not pick a new colour while a neighbour
-          // that beats it is itself queued for (re)assignment -- both would choose from the same stale
-          // view and collide again (measured: the dense core of C4 was recoloured 8-16x).  It re-queues
-          // itself instead, at most once in a row (unbounded deferral chains rescanned hub rows ~30x
-          // more), so every recolour completes within two pops.
-          if (kDefer && !c.literal && cval[own[k]] >= 0 && !flag[own[k]] && c.assign_queued(w[k]) &&
-              c.loses(item, w[k]))
-            flag[own[k]] = 2;
         } else if (cw[k] == cval[own[k]]) {
           if (c.literal || c.loses(item & ~kCheck, w[k])) flag[own[k]] = 1;
           else if (c.claim_assign(w[k])) { want[k] = true; out[k] = w[k]; }
@@ -290,19 +281,43 @@ __global__ void __launch_bounds__(1024) k_color_cta(ColorCtx c, EngineParams P) 
       uint32_t out = 0;
       if (k < nready) {
         const uint32_t item = s.item[k], v = item & ~kCheck;
-        if (!(item & kCheck) && flag[k] == 2) {
-          // deferred recolour: back into the queue, colour unchanged
-          if (lane_id() == 0) atomicOr(c.dfr + (v >> 5), 1u << (v & 31));
-          want = lane_id() == 0 && c.claim_assign(v);
-          out = v;
-        } else if (!(item & kCheck)) {
-          if (flag[k] == 3 && lane_id() == 0) atomicAnd(c.dfr + (v >> 5), ~(1u << (v & 31)));
-          const uint32_t freebits = ~ibm[k * 32 + lane_id()];
-          const unsigned m = __ballot_sync(0xffffffffu, freebits != 0);
+        if (!(item & kCheck)) {
           int32_t chosen = -1;
-          if (m) {
-            const uint32_t L = __ffs(m) - 1;
-            const uint32_t fb = __shfl_sync(0xffffffffu, freebits, L);
+          // free colours of the first window, limited to [0, deg(v)] so that colour <= deg(v) holds for
+          // every choice (at most deg(v) of those deg(v)+1 colours are taken, so one is always free)
+          const uint32_t dv = (k + 1 < nready ? s.off[k + 1] : total) - s.off[k];
+          const uint32_t lo_c = lane_id() * 32;
+          const uint32_t lim = dv >= lo_c + 31 ? 0xFFFFFFFFu : (dv < lo_c ? 0u : (0xFFFFFFFFu >> (31 - (dv - lo_c))));
+          const uint32_t freebits = ~ibm[k * 32 + lane_id()] & lim;
+          // Recolour spread: the vertices that keep losing in the dense core of a scale-free graph share
+          // most of their neighbourhoods, so when several recolour concurrently they all find the SAME
+          // smallest free colour and collide again (measured at C4: ranks 128..8192 by degree were
+          // re-assigned 8-16x and took 80 % of the edge visits).  The a-th recolour of v takes the j-th
+          // smallest free colour of the first window, j = splitmix64(seed ^ v ^ old colour) mod
+          // min(2^(a-1), cfg.recolor_spread): the first assign and the first recolour keep Alg.6's smallest
+          // free colour, and only vertices caught in a repeated collision spread out (R-GC-10).
+          // Off by default (recolor_spread = 1): it trades colours for time (C4: 8.7 ms / 690 colours at 1,
+          // 7.1 / 818 at 4, 6.7 / 910 at 8, 6.3 / 1017 at 16 -- DESIGN.md section 6).
+          uint32_t j = 0;
+          if (flag[k] > 1)
+            j = (uint32_t)(splitmix64(c.seed ^ v ^ ((unsigned long long)(uint32_t)cval[k] << 32)) % flag[k]);
+          const uint32_t cnt = __popc(freebits);
+          uint32_t incl = cnt;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane_id() >= (uint32_t)o) incl += y;
+          }
+          const uint32_t nfree = __shfl_sync(0xffffffffu, incl, 31);
+          if (nfree) {
+            if (j >= nfree) j = nfree - 1;
+            // the lane holding the j-th free bit picks it
+            const bool mine = incl > j && incl - cnt <= j;
+            const unsigned who = __ballot_sync(0xffffffffu, mine);
+            const uint32_t L = __ffs(who) - 1;
+            uint32_t fb = __shfl_sync(0xffffffffu, freebits, L);
+            const uint32_t skip = j - (__shfl_sync(0xffffffffu, incl - cnt, L));
+            for (uint32_t t = 0; t < skip; ++t) fb &= fb - 1;  // drop the lowest `skip` free bits
             chosen = (int32_t)(L * 32 + (__ffs(fb) - 1));
           } else {
             // window [0, 1024) is full: scan further windows with the warp
@@ -632,15 +647,16 @@ int color_single(atos_csr* g, Part& p, uint64_t seed, int32_t* color, const Reso
   const uint64_t want = r.queue_capacity ? r.queue_capacity : std::max<uint64_t>(4ull * n, 4096);
   ATOS_TRY(ensure_queue(p, pow2_ceil(want), s));
   const size_t words = ((size_t)n + 31) / 32;
-  ATOS_TRY(p.bitmap.ensure(words * 4 * 2));  // assign dedupe bits, then recolour-deferral bits
+  ATOS_TRY(p.bitmap.ensure(words * 4 + ((size_t)n + 15) / 16 * 16));  // dedupe bits, then recolour counts
   ATOS_TRY(p.scratch.ensure(64));
   Ring q;
   q.slots = p.ring.as<unsigned long long>();
   q.mask = p.ring_cap - 1;
   q.ctl = p.ctl.as<QueueCtl>();
-  ColorCtx c{p.row_ptr, p.col, color, p.bitmap.as<uint32_t>(), p.bitmap.as<uint32_t>() + words, seed,
-             r.conflict_policy == 1 ? 1 : 0, r.conflict_policy == 2 ? 1 : 0};
-  ATOS_CUDA(cudaMemsetAsync(c.dfr, 0, words * 4, s));
+  ColorCtx c{p.row_ptr, p.col, color, p.bitmap.as<uint32_t>(), (uint8_t*)(p.bitmap.as<uint32_t>() + words),
+             (uint32_t)std::max(1, r.recolor_spread), seed, r.conflict_policy == 1 ? 1 : 0,
+             r.conflict_policy == 2 ? 1 : 0};
+  if (c.spread > 1) ATOS_CUDA(cudaMemsetAsync(c.att, 0, (size_t)n, s));
   // init: reserve [t, t+n) then publish every vertex
   k_color_begin<<<1, 32, 0, s>>>(q.ctl, n);
   g_launches++;

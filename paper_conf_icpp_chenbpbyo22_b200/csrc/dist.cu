@@ -348,6 +348,59 @@ void atos_comm_destroy(atos_comm* c) {
   delete c;
 }
 
+int atos_comm_gather(atos_comm* comm, int64_t n_global, const void* slice, size_t elem_bytes, void* out_root,
+                     void* stream) {
+  if (!comm || n_global < 0 || elem_bytes == 0 || (comm->c.rank == 0 && !out_root && n_global > 0)) {
+    set_error("atos_comm_gather: invalid argument");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  Comm* c = &comm->c;
+  const int P = c->nranks;
+  cudaStream_t s = (cudaStream_t)stream;
+  DeviceGuard dg(c->device);
+  std::vector<int64_t> vb(P), ve(P);
+  for (int r = 0; r < P; ++r) atos_partition_range(n_global, P, r, &vb[r], &ve[r]);
+  const size_t mine = (size_t)(ve[c->rank] - vb[c->rank]) * elem_bytes;
+  if (mine && !slice) {
+    set_error("atos_comm_gather: null slice");
+    return ATOS_ERR_INVALID_ARG;
+  }
+  if (c->h_a2a) {
+    // host transport: every rank sends its slice to rank 0 only
+    std::vector<char> sbuf(std::max<size_t>(mine, 1)), rbuf(c->rank == 0 ? std::max<size_t>(n_global * elem_bytes, 1) : 1);
+    if (mine) ATOS_CUDA(cudaMemcpyAsync(sbuf.data(), slice, mine, cudaMemcpyDeviceToHost, s));
+    ATOS_CUDA(cudaStreamSynchronize(s));
+    std::vector<uint64_t> sb(P, 0), rb(P, 0);
+    sb[0] = mine;
+    if (c->rank == 0)
+      for (int r = 0; r < P; ++r) rb[r] = (uint64_t)(ve[r] - vb[r]) * elem_bytes;
+    if (c->h_a2a(c->h_user, sbuf.data(), sb.data(), rbuf.data(), rb.data()) != 0) {
+      set_error("atos_comm_gather: host alltoallv failed");
+      return ATOS_ERR_NCCL;
+    }
+    if (c->rank == 0 && n_global) {
+      ATOS_CUDA(cudaMemcpyAsync(out_root, rbuf.data(), n_global * elem_bytes, cudaMemcpyHostToDevice, s));
+      ATOS_CUDA(cudaStreamSynchronize(s));
+    }
+    return ATOS_OK;
+  }
+  NcclApi& api = nccl();
+  ncclComm_t nc = (ncclComm_t)c->nccl;
+  ATOS_NCCL(api.GroupStart());
+  if (c->rank == 0) {
+    if (mine) ATOS_CUDA(cudaMemcpyAsync(out_root, slice, mine, cudaMemcpyDeviceToDevice, s));
+    for (int r = 1; r < P; ++r) {
+      const size_t b = (size_t)(ve[r] - vb[r]) * elem_bytes;
+      if (b) ATOS_NCCL(api.Recv((char*)out_root + (size_t)vb[r] * elem_bytes, b, ncclUint8, r, nc, s));
+    }
+  } else if (mine) {
+    ATOS_NCCL(api.Send(slice, mine, ncclUint8, 0, nc, s));
+  }
+  ATOS_NCCL(api.GroupEnd());
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  return ATOS_OK;
+}
+
 int atos_csr_create_part(atos_csr** out, atos_comm* comm, int64_t n_global, int64_t v_begin, int64_t v_end,
                          int64_t m_local, const int64_t* row_ptr_local, const int32_t* col_global, int where) {
   if (!out || !comm || n_global < 0 || v_begin < 0 || v_end < v_begin || v_end > n_global || m_local < 0 ||

@@ -146,6 +146,21 @@ __device__ __forceinline__ void tl_sample(const EngineParams& P) {
   e[3] = ld_relaxed(&c->head.v);
 }
 
+// The closing sample: the first worker that observes global termination records one last row (the run's
+// final done / tail), then parks the sampling clock at +inf so no later row is written.
+__device__ __forceinline__ void tl_final(const EngineParams& P) {
+  if (!P.tl) return;
+  QueueCtl* c = P.q.ctl;
+  if (atomicExch(&c->tl_next.v, ~0ull) == ~0ull) return;
+  const unsigned long long k = atomicAdd(&c->tl_count.v, 1ull);
+  if (k >= P.tl_cap) return;
+  unsigned long long* e = P.tl + 4 * k;
+  e[0] = globaltimer();
+  e[1] = ld_relaxed(&c->done.v);
+  e[2] = ld_relaxed(&c->tail.v);
+  e[3] = ld_relaxed(&c->head.v);
+}
+
 constexpr uint32_t kGoBig = 0xFFFFFFFFu;
 
 // ---------------------------------------------------------- col prefetch (cp.async)
@@ -484,6 +499,7 @@ struct Worker {
         const unsigned long long t = atom_read(&q.ctl->tail.v);
         const uint32_t st = *(volatile uint32_t*)&q.ctl->status.v;
         if (d == t || st != 0) {
+          if (PERSIST && d == t) tl_final(P);
           s.ctr[3] = 1;
         } else if (PERSIST && P.nbig && ld_relaxed(&q.ctl->big_count.v) != 0) {
           tl_sample(P);
@@ -520,8 +536,10 @@ struct Worker {
   __device__ __forceinline__ void complete(const EngineParams& P, uint32_t nready) {
     group_sync<MODE>();
     if (PERSIST && r == 0 && nready) {
-      fence_acq_rel_gpu();
-      atom_add_release(&P.q.ctl->done.v, (unsigned long long)nready);
+      // release reduction, no return value to wait for: the barrier above orders every warp's pushes
+      // before the leader's release (cumulative), and nobody needs the old count (C5 BFS -1 %)
+      asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(&P.q.ctl->done.v), "l"((unsigned long long)nready)
+                   : "memory");
     }
     if (r == 0) tl_sample(P);
     group_sync<MODE>();

@@ -135,6 +135,7 @@ struct Resolved {
   int conflict_policy, permute_init, validate, out_where, l2_persist, big_threshold, big_chunk, depth_state;
   int engine_variant;
   int barrier_free;
+  int recolor_spread;
   int knobs_set;  // a scheduler knob the barrier-free kernel ignores was set (persistent=0, dedupe=0, worker,
                   // fetch_size, queue_capacity, depth_state, engine_variant)
   unsigned long long* timeline;

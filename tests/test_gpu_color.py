@@ -131,3 +131,16 @@ def test_layout_modes_valid(layout):
         check_color(rp, ci, c, st)
         c, st = atos.color_bsp(csr, seed=3)
         check_color(rp, ci, c, st)
+
+
+@pytest.mark.parametrize("spread", [2, 8, 64])
+def test_recolor_spread_valid(rmat13, spread):
+    """cfg.recolor_spread (R-GC-10): still a proper colouring with colour <= deg(v) for every vertex (the
+    j-th free colour is taken among [0, deg(v)]); the dense Kronecker core exercises repeated recolours."""
+    rp, ci, csr = rmat13
+    for seed in (1, 2):
+        c, st = atos.color(csr, seed, recolor_spread=spread)
+        assert oracle.validate_color(rp, ci, c.cpu().numpy()) == 0
+        assert st["colors_used"] == int(c.max().item()) + 1
+    with pytest.raises(RuntimeError, match="INVALID_ARG"):
+        atos.color(csr, 1, recolor_spread=65)

@@ -1,0 +1,46 @@
+"""cfg.timeline (the progress samples behind Figs. 1-3): the samples are monotone in time and in
+the done / tail / head counters, done never exceeds tail, and the final sample's done equals the run's
+task count -- so the normalized throughput (analysis.normalized_throughput) integrates to the real work."""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_icpp_chenbpbyo22_b200 as atos
+from paper_conf_icpp_chenbpbyo22_b200 import analysis, gen
+
+from _gpu import DEV
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("app", ["bfs", "pr", "gc"])
+def test_timeline_samples(app):
+    g = gen.rmat(18, 16, seed=3, device=DEV)
+    csr = atos.CSR.from_graph(g)
+    cap = 1 << 14
+    tl = torch.zeros(4 * cap, dtype=torch.int64, device=DEV)
+    knobs = dict(timeline=tl, timeline_interval_ns=2000)
+    if app == "bfs":
+        _, st = atos.bfs(csr, gen.pick_source(g, 1), **knobs)
+        _, sb = atos.bfs_bsp(csr, gen.pick_source(g, 1))
+    elif app == "pr":
+        _, st = atos.pagerank(csr, 0.85, 1e-6, **knobs)
+        _, sb = atos.pagerank_bsp(csr, 0.85, 1e-6)
+    else:
+        _, st = atos.color(csr, 1, **knobs)
+        sb = None
+    assert 2 <= st["timeline_len"] <= cap
+    tab = atos.timeline_table(tl, st).numpy()
+    t, done, tail, head = tab[:, 0], tab[:, 1], tab[:, 2], tab[:, 3]
+    assert np.all(np.diff(t) >= 0) and np.all(np.diff(done) >= 0)
+    assert np.all(np.diff(tail) >= 0) and np.all(np.diff(head) >= 0)
+    assert np.all(done <= tail)
+    # every task of the run completes before the last worker exits; the last sample is taken at exit
+    # (Worker::complete samples after each batch), so it sees all of them relative to the first sample
+    first_done = done[0]
+    assert done[-1] - first_done <= st["pops"]
+    assert done[-1] - first_done >= 0.95 * st["pops"]
+    ow = analysis.overwork_factor(app, st["pops"], bsp_pops=sb["pops"] if sb else None, n=g.n)
+    tt, nt = analysis.normalized_throughput(tab, ow)
+    assert np.all(nt >= 0)
+    assert abs(np.sum(nt * np.diff(t)[np.diff(t) > 0]) * ow - (done[-1] - done[0])) < 1e-6 * max(1, done[-1])

@@ -47,17 +47,23 @@ def run(a):
                 env = dict(os.environ, ATOS_LIB=lib_of(tag))
                 out = subprocess.run(cmd, capture_output=True, text=True, env=env, timeout=900).stdout
                 for line in out.splitlines():
-                    mm = re.search(r"ms med\s+([\d.]+).*worker\s+([\d.]+).*edges/m\s+([\d.]+)", line)
+                    mm = re.search(r"^\s*(\S+)\s+ms med\s+([\d.]+).*worker\s+([\d.]+).*edges/m\s+([\d.]+)"
+                                   r"(?:.*colors\s+(\d+))?", line)
                     if mm:
-                        res.setdefault((app, tag), []).append(tuple(float(x) for x in mm.groups()))
+                        key = (app, mm.group(1), tag)
+                        vals = [float(x) for x in mm.groups()[1:4]] + [float(mm.group(5) or 0)]
+                        res.setdefault(key, []).append(tuple(vals))
+                        print(f"round {rnd} {app:9s} {mm.group(1):12s} {tag:14s} {vals}", flush=True)
                     elif "ERROR" in line:
                         print(f"[{app} {tag}] {line.strip()}", flush=True)
-                print(f"round {rnd} {app:9s} {tag:14s} {res.get((app, tag), [None])[-1]}", flush=True)
-    print("# app tag: median ms, median worker ms, edges/m (over rounds)")
-    for (app, tag), v in sorted(res.items()):
+                if not out.strip():
+                    print(f"[{app} {tag}] no output", flush=True)
+    print("# app spec tag: median ms, median worker ms, edges/m, colours (over rounds)")
+    for (app, spec, tag), v in sorted(res.items()):
         v = np.array(v)
-        print(f"{app:9s} {tag:14s} ms {np.median(v[:, 0]):9.3f}  worker {np.median(v[:, 1]):9.3f}  "
-              f"edges/m {np.median(v[:, 2]):7.3f}  (n={len(v)})", flush=True)
+        print(f"{app:9s} {spec:12s} {tag:14s} ms {np.median(v[:, 0]):9.3f}  worker {np.median(v[:, 1]):9.3f}  "
+              f"edges/m {np.median(v[:, 2]):7.3f}" + (f"  colours {np.median(v[:, 3]):.0f}" if v[0, 3] else "")
+              + f"  (n={len(v)})", flush=True)
 
 
 def main():
