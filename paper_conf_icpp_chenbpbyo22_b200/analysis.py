@@ -28,8 +28,8 @@ def overwork_factor(app: str, pops: int, bsp_pops: int | None = None, n: int | N
 
 def throughput_series(table) -> tuple[np.ndarray, np.ndarray]:
     """(t_us at interval mid-points, tasks completed per microsecond) from a timeline table
-    (rows: t_us since the first sample, done, tail, head -- see timeline_table())."""
-    t = np.asarray(table[:, 0], dtype=np.float64)
+    (rows: globaltimer ns since the first sample, done, tail, head -- see timeline_table())."""
+    t = np.asarray(table[:, 0], dtype=np.float64) / 1e3
     done = np.asarray(table[:, 1], dtype=np.float64)
     if t.size < 2:
         return np.zeros(0), np.zeros(0)

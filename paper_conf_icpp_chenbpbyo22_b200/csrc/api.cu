@@ -7,6 +7,7 @@
 #include <thread>
 #include <algorithm>
 #include <functional>
+#include <unordered_map>
 
 #include "internal.h"
 
@@ -54,13 +55,46 @@ int pool_of(int dev, PoolOf** out) {
 }
 }  // namespace
 
+// Block cache on top of the pool: freed blocks are kept by exact size class, so a handle created and
+// destroyed per step gets the same blocks back without the pool re-mapping memory (measured: the pool
+// alone still cost 20-55 ms on some steps when a multi-GB request no longer fit its split blocks).
+namespace {
+struct CacheEnt {
+  void* p;
+  size_t bytes;
+  int dev;
+};
+std::mutex g_cache_mu;
+std::vector<CacheEnt> g_cache;                       // free blocks, oldest first
+std::unordered_map<void*, std::pair<size_t, int>> g_live;  // every library block: size, device
+size_t g_cache_bytes = 0;
+constexpr size_t kCacheCap = 48ull << 30;
+}  // namespace
+
 int dev_alloc(void** p, size_t bytes) {
   *p = nullptr;
   int dev = 0;
   ATOS_CUDA(cudaGetDevice(&dev));
+  if (!bytes) bytes = 16;
+  {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    size_t best = (size_t)-1;
+    for (size_t i = 0; i < g_cache.size(); ++i) {
+      const CacheEnt& c = g_cache[i];
+      if (c.dev == dev && c.bytes >= bytes && c.bytes <= bytes + bytes / 4 &&
+          (best == (size_t)-1 || c.bytes < g_cache[best].bytes))
+        best = i;
+    }
+    if (best != (size_t)-1) {
+      *p = g_cache[best].p;
+      g_cache_bytes -= g_cache[best].bytes;
+      g_cache.erase(g_cache.begin() + best);
+      return ATOS_OK;
+    }
+  }
   PoolOf* P = nullptr;
   ATOS_TRY(pool_of(dev, &P));
-  cudaError_t e = cudaMallocFromPoolAsync(p, bytes ? bytes : 16, P->pool, P->s);
+  cudaError_t e = cudaMallocFromPoolAsync(p, bytes, P->pool, P->s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(P->s);  // usable by every stream from here on
   if (e != cudaSuccess) {
     *p = nullptr;
@@ -68,20 +102,42 @@ int dev_alloc(void** p, size_t bytes) {
     set_error("device allocation of %zu bytes failed: %s", bytes, cudaGetErrorString(e));
     return e == cudaErrorMemoryAllocation ? ATOS_ERR_OOM : ATOS_ERR_CUDA;
   }
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  g_live[*p] = {bytes, dev};
   return ATOS_OK;
 }
 
 void dev_free(void* p) {
   if (!p) return;
+  size_t bytes = 0;
   int dev = 0;
-  cudaPointerAttributes a;
-  if (cudaPointerGetAttributes(&a, p) == cudaSuccess) dev = a.device;
-  else cudaGetLastError();
-  PoolOf* P = nullptr;
-  if (pool_of(dev, &P) != ATOS_OK) return;
+  {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    auto it = g_live.find(p);
+    if (it == g_live.end()) return;  // not ours
+    bytes = it->second.first;
+    dev = it->second.second;
+  }
   DeviceGuard dg(dev);
   cudaDeviceSynchronize();  // no kernel may still use the block (cudaFree's own guarantee)
-  cudaFreeAsync(p, P->s);
+  std::vector<CacheEnt> evict;
+  {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    g_cache.push_back({p, bytes, dev});
+    g_cache_bytes += bytes;
+    while (g_cache_bytes > kCacheCap && !g_cache.empty()) {
+      evict.push_back(g_cache.front());
+      g_cache_bytes -= g_cache.front().bytes;
+      g_live.erase(g_cache.front().p);
+      g_cache.erase(g_cache.begin());
+    }
+  }
+  for (const CacheEnt& c : evict) {
+    PoolOf* P = nullptr;
+    if (pool_of(c.dev, &P) != ATOS_OK) continue;
+    DeviceGuard dg2(c.dev);
+    cudaFreeAsync(c.p, P->s);
+  }
   cudaGetLastError();
 }
 
@@ -300,6 +356,16 @@ void set_l2_window(cudaStream_t s, void* base, size_t bytes, bool on) {
   }
   cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
   cudaGetLastError();  // best effort
+}
+
+void trace_mark(const char* what, bool sync) {
+  static const bool on = getenv("ATOS_TRACE") != nullptr;
+  if (!on) return;
+  static thread_local std::chrono::steady_clock::time_point last = std::chrono::steady_clock::now();
+  if (sync) cudaDeviceSynchronize();
+  const auto now = std::chrono::steady_clock::now();
+  fprintf(stderr, "[atos trace] %-28s %9.3f ms\n", what, std::chrono::duration<double, std::milli>(now - last).count());
+  last = now;
 }
 
 int stream_wait(cudaStream_t s, double timeout_s) {
@@ -529,9 +595,11 @@ int run_with_output(atos_csr* g, T* out, int64_t len, const Resolved& r, DevBuf&
     rm.map_done = nullptr;
     ATOS_TRY(rc);
     if (!mapped) ATOS_TRY(layout_scatter<T>(g, staging.as<T>(), dst, r.stream));
+    trace_mark("output: device", true);
     if (r.out_where != ATOS_MEM_DEVICE) {
       ATOS_CUDA(cudaMemcpyAsync(out, dst, (size_t)len * sizeof(T), cudaMemcpyDeviceToHost, r.stream));
       ATOS_CUDA(cudaStreamSynchronize(r.stream));
+      trace_mark("output: D2H", true);
     }
     return ATOS_OK;
   }

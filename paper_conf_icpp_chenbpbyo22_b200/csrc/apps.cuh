@@ -59,6 +59,7 @@ template <bool PART, bool ACQ = true>
 struct BfsAppT {
   static constexpr bool kAcquirePop = ACQ;
   static constexpr bool kPfCta = false;  // CTA workers other than the (256,5) build: direct col loads
+  static constexpr bool kFusedBegin = false;
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
   const uint32_t* __restrict__ row_ptr;
@@ -172,6 +173,10 @@ struct BfsByteAppT {
   // ordering through the address dependency alone); the AND itself can then stay relaxed.
   static constexpr bool kAcquirePop = true;
   static constexpr bool kPfCta = false;
+#ifndef ATOS_FUSED_BEGIN
+#define ATOS_FUSED_BEGIN 1
+#endif
+  static constexpr bool kFusedBegin = ATOS_FUSED_BEGIN != 0 && !PART;  // consume_slot_fused (engine.cuh)
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // the 32-bit word holding w's state byte (prefilter and CAS guess)
   const uint32_t* __restrict__ row_ptr;
@@ -280,6 +285,7 @@ struct PrAppT {
 #define ATOS_PF_PR 1
 #endif
   static constexpr bool kPfCta = ATOS_PF_PR != 0 && !PART;  // cp.async col prefetch (C3: 65.3 -> 63.6 ms)
+  static constexpr bool kFusedBegin = false;  // begin() takes the residue: not speculatable
   using Payload = double;  // delta = alpha * rho / deg(v)
   using Token = double;    // residue before our atomicAdd
   const uint32_t* __restrict__ row_ptr;

@@ -28,6 +28,8 @@
 //   const uint32_t* col;  (neighbour array)
 //   bool sweep(...) hooks are app-specific and live in the app files.
 #pragma once
+#include <type_traits>
+
 #include "device.cuh"
 
 namespace atos {
@@ -370,6 +372,40 @@ __device__ __forceinline__ void consume_slot(const Ring& q, const GroupSmem<Payl
   }
 }
 
+// Fused consume + begin (apps with kFusedBegin, the byte-state BFS): after the acquire load has shown the
+// slot published, the slot-freeing CAS (relaxed: the acquire load already synchronised with the
+// producer's release) and the app's begin (row_ptr loads, the state RMW) are issued together, so a pop
+// costs two dependent round trips instead of three.  If the CAS loses (a lapping producer stole the item,
+// which the default capacity makes impossible in practice) the item is dropped; the speculative begin is
+// then harmless for BFS: clearing the queued flag early can only cause a duplicate push of the vertex,
+// and BFS is label-correcting.
+template <class App>
+__device__ __forceinline__ void consume_slot_fused(const Ring& q, const GroupSmem<typename App::Payload>& s,
+                                                   unsigned long long idx, const App& app) {
+  unsigned long long* slot = q.slots + (idx & q.mask);
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(slot) : "memory");
+  const int32_t d = (int32_t)((uint32_t)(v >> 32) - (uint32_t)(idx + 1));
+  if (d < 0) {
+    const uint32_t k = atomicAdd(&s.ctr[2], 1u);
+    s.pend2[k] = idx;
+    return;
+  }
+  if (d > 0) return;
+  const uint32_t item = (uint32_t)v;
+  const unsigned long long freed = make_slot(idx + q.mask + 1, 0u);
+  const unsigned long long old = atomicCAS(slot, v, freed);
+  uint32_t st = 0, dg = 0;
+  typename App::Payload p{};
+  if (!app.begin(item, st, dg, p)) dg = 0;
+  if (old != v) return;
+  const uint32_t k = atomicAdd(&s.ctr[0], 1u);
+  s.item[k] = item;
+  s.start[k] = st;
+  s.off[k] = dg;
+  s.pay[k] = p;
+}
+
 // ------------------------------------------------------------ worker group
 // One worker (a CTA, a warp, or -- for MODE_THREAD -- a warp of 32 thread
 // workers that share one claim) and its queue protocol: claim / gather /
@@ -410,7 +446,9 @@ struct Worker {
 
   // Returns the number of ready items now in s.item[0..n), or 0 when the
   // worker must exit (global termination, watchdog, or end of a discrete chunk).
-  __device__ __forceinline__ uint32_t acquire(const EngineParams& P) {
+  // With a fused app (kFusedBegin) the items' begin() results are already in s.start / s.off / s.pay.
+  template <class FusedApp = void>
+  __device__ __forceinline__ uint32_t acquire(const EngineParams& P, const FusedApp* fapp = nullptr) {
     const Ring& q = P.q;
     while (true) {
       // ------------------------------------------------------ 1. claim
@@ -476,8 +514,13 @@ struct Worker {
       {
         const unsigned long long cb = *(unsigned long long*)&s.ctr[6];
         const uint32_t cc = s.ctr[4], np = s.ctr[1];
-        for (uint32_t i = r; i < cc; i += G) consume_slot<ACQ>(q, s, cb + i);
-        for (uint32_t i = r; i < np; i += G) consume_slot<ACQ>(q, s, s.pend[i]);
+        if constexpr (!std::is_void<FusedApp>::value) {
+          for (uint32_t i = r; i < cc; i += G) consume_slot_fused(q, s, cb + i, *fapp);
+          for (uint32_t i = r; i < np; i += G) consume_slot_fused(q, s, s.pend[i], *fapp);
+        } else {
+          for (uint32_t i = r; i < cc; i += G) consume_slot<ACQ>(q, s, cb + i);
+          for (uint32_t i = r; i < np; i += G) consume_slot<ACQ>(q, s, s.pend[i]);
+        }
       }
       group_sync<MODE>();
       const uint32_t nready = s.ctr[0];
@@ -649,14 +692,21 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
       group_sync<MODE>();
       ATOS_PH(PH_BIG);
     }
-    const uint32_t nready = wk.acquire(P);
+    constexpr bool kFused = App::kFusedBegin && MODE == MODE_CTA;
+    const uint32_t nready = kFused ? wk.acquire(P, &app) : wk.acquire(P);
     if (nready == kGoBig) continue;
     if (nready == 0) break;
     // ---------------------------------------------------------- begin (per item)
     for (uint32_t k = r; k < nready; k += G) {
       uint32_t st = 0, dg = 0;
       Payload p{};
-      if (!app.begin(s.item[k], st, dg, p)) dg = 0;
+      if (kFused) {
+        st = s.start[k];
+        dg = s.off[k];
+        p = s.pay[k];
+      } else if (!app.begin(s.item[k], st, dg, p)) {
+        dg = 0;
+      }
       if (assist && dg > P.big_threshold && register_big(P, s.item[k], st, dg, p)) {
         dg = 0;  // expanded by the assist chunks; counted done by the last chunk
         atomicAdd(&s.ctr[5], 1u);

@@ -208,6 +208,10 @@ struct WorkerTimer {
   }
 };
 
+// Host-side phase tracer (tools: ATOS_TRACE=1): prints the wall time since the previous mark of this
+// thread; `sync` first waits for the device so the time covers the enqueued work.
+void trace_mark(const char* what, bool sync = false);
+
 // wait for the stream, honouring cfg.timeout_s (polling) -- returns ATOS_ERR_TIMEOUT on expiry
 int stream_wait(cudaStream_t s, double timeout_s);
 

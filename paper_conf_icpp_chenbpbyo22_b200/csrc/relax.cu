@@ -357,6 +357,7 @@ static int bfs_single_bytes(Part& p, int64_t src, uint32_t* depth, const Resolve
   ATOS_TRY(p.shadow.ensure(nb));
   uint8_t* state = p.shadow.as<uint8_t>();
   ATOS_CUDA(cudaMemsetAsync(state, (int)kBUnreached, nb, s));
+  trace_mark("bfs: state", true);
   Ring q = ring_of(p);
   k_bfs_byte_init<<<1, 32, 0, s>>>(state, q, (uint32_t)src, r.watchdog_ns);
   g_launches++;
@@ -365,6 +366,7 @@ static int bfs_single_bytes(Part& p, int64_t src, uint32_t* depth, const Resolve
   BfsByteApp app{p.row_ptr, p.col, state, (uint32_t*)&q.ctl->status.v, 0ull, 0ull};
   p.ring_clean = false;
   int rc = launch_relax(app, q, r, p, st);
+  trace_mark("bfs: worker", true);
   if (r.l2_persist) set_l2_window(s, nullptr, 0, false);
   if (rc != ATOS_OK) return rc;
   ATOS_TRY(finish_queue(p, s, st, "bfs"));
@@ -388,7 +390,9 @@ int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolve
   const int64_t n = p.n_local;
   uint64_t want = r.queue_capacity ? r.queue_capacity : (uint64_t)std::max<int64_t>(2 * n, 1024);
   if (!r.dedupe && !r.queue_capacity) want = (uint64_t)std::max<int64_t>(4 * n, 4096);
+  trace_mark("bfs: enter", true);
   ATOS_TRY(ensure_queue(p, pow2_at_least(want), s));
+  trace_mark("bfs: ensure_queue", true);
   // byte state first (dedupe mode); a traversal deeper than 125 levels re-runs with u32 words
   if (r.dedupe && r.depth_state != 2) {
     bool deep = false;

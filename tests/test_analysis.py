@@ -8,7 +8,7 @@ from paper_conf_icpp_chenbpbyo22_b200 import analysis
 def test_throughput_series_constant_rate():
     t = np.arange(0, 100, 5.0)
     done = 3.0 * t  # 3 tasks per microsecond
-    tab = np.stack([t, done, done + 10, done], axis=1)
+    tab = np.stack([t * 1e3, done, done + 10, done], axis=1)  # timeline rows carry nanoseconds
     mid, tp = analysis.throughput_series(tab)
     np.testing.assert_allclose(mid, t[1:] - 2.5)
     np.testing.assert_allclose(tp, 3.0)
@@ -17,7 +17,7 @@ def test_throughput_series_constant_rate():
 
 
 def test_normalized_divides_by_overwork_and_skips_repeated_timestamps():
-    tab = np.array([[0, 0, 0, 0], [10, 100, 0, 0], [10, 100, 0, 0], [30, 300, 0, 0]], dtype=np.float64)
+    tab = np.array([[0, 0, 0, 0], [10e3, 100, 0, 0], [10e3, 100, 0, 0], [30e3, 300, 0, 0]], dtype=np.float64)
     t, nt = analysis.normalized_throughput(tab, 2.0)
     np.testing.assert_allclose(t, [5.0, 20.0])
     np.testing.assert_allclose(nt, [5.0, 5.0])

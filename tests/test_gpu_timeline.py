@@ -43,4 +43,5 @@ def test_timeline_samples(app):
     ow = analysis.overwork_factor(app, st["pops"], bsp_pops=sb["pops"] if sb else None, n=g.n)
     tt, nt = analysis.normalized_throughput(tab, ow)
     assert np.all(nt >= 0)
-    assert abs(np.sum(nt * np.diff(t)[np.diff(t) > 0]) * ow - (done[-1] - done[0])) < 1e-6 * max(1, done[-1])
+    dt_us = np.diff(t)[np.diff(t) > 0] / 1e3
+    assert abs(np.sum(nt * dt_us) * ow - (done[-1] - done[0])) < 1e-6 * max(1, done[-1])

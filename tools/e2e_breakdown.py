@@ -16,7 +16,7 @@ t = time.perf_counter(); x = torch.empty_like(ci, device="cuda"); x.copy_(ci); t
 print(f"raw H2D of col ({ci.numel() * 4 / 1e9:.2f} GB): {1e3 * (time.perf_counter() - t):.1f} ms")
 del x
 torch.cuda.empty_cache()
-for k in range(4):
+for k in range(int(os.environ.get("E2E_STEPS", "4"))):
     t0 = time.perf_counter()
     csr = atos.CSR(rp, ci, device=0)
     t1 = time.perf_counter()

@@ -51,7 +51,7 @@ def main():
     print("#   t_ms   tasks/us  normalized/us")
     idx = sorted(set(int(i * (len(t) - 1) / max(1, a.rows - 1)) for i in range(a.rows))) if len(t) else []
     for i in idx:
-        print(f"{t[i] / 1e3:8.3f} {tp[i]:10.2f} {nt[i]:10.2f}")
+        print(f"{t[i] / 1e3:8.3f} {tp[i]:10.1f} {nt[i]:10.1f}")
 
 
 if __name__ == "__main__":
