@@ -566,6 +566,12 @@ void destroy_part(Part& p) {
                     &p.nb_peers};
   for (DevBuf* b : bufs) b->release();
   pinned_page_release(p.host_pinned);
+  for (void* b : p.nb_peer_base)
+    if (b) cudaIpcCloseMemHandle(b);
+  p.nb_peer_base.clear();
+  if (p.nb_ipc) cudaFree(p.nb_ipc);
+  p.nb_ipc = nullptr;
+  p.nb_ipc_bytes = 0;
   p.host_pinned = nullptr;
 }
 
@@ -737,11 +743,13 @@ int atos_bfs(const atos_csr* gc, int64_t src, uint32_t* depth_out, const atos_cf
   CallTimer tm(r.stream);
   int rc;
   if (r.barrier_free) {
-    if (g->comm || g->num_parts < 2) {
-      set_error("atos_bfs: barrier_free needs a loopback-partitioned graph (num_parts > 1, one process)");
+    if (!g->comm && g->num_parts < 2) {
+      set_error("atos_bfs: barrier_free needs a partitioned graph (loopback num_parts > 1, or one partition per "
+                "process)");
       return ATOS_ERR_UNSUPPORTED;
     }
-    rc = run_with_output<uint32_t>(g, depth_out, g->n, r, g->parts[0].vbuf_c,
+    const int64_t len = g->comm ? g->parts[0].n_local : g->n;
+    rc = run_with_output<uint32_t>(g, depth_out, len, r, g->parts[0].vbuf_c,
                                    [&](uint32_t* d) { return bfs_nobarrier(g, src, d, r, st); });
   } else if (g->comm || g->num_parts > 1) {
     const int64_t len = g->comm ? g->parts[0].n_local : g->n;
@@ -784,11 +792,13 @@ int atos_pagerank(const atos_csr* gc, double alpha, double eps, double* rank_out
   int rc;
   if (g->n == 0) return ATOS_OK;
   if (r.barrier_free) {
-    if (g->comm || g->num_parts < 2) {
-      set_error("atos_pagerank: barrier_free needs a loopback-partitioned graph (num_parts > 1, one process)");
+    if (!g->comm && g->num_parts < 2) {
+      set_error("atos_pagerank: barrier_free needs a partitioned graph (loopback num_parts > 1, or one partition "
+                "per process)");
       return ATOS_ERR_UNSUPPORTED;
     }
-    rc = run_with_output<double>(g, rank_out, g->n, r, g->parts[0].vbuf_c,
+    const int64_t len = g->comm ? g->parts[0].n_local : g->n;
+    rc = run_with_output<double>(g, rank_out, len, r, g->parts[0].vbuf_c,
                                  [&](double* d) { return pagerank_nobarrier(g, alpha, eps, d, r, st); });
   } else if (g->comm || g->num_parts > 1) {
     const int64_t len = g->comm ? g->parts[0].n_local : g->n;

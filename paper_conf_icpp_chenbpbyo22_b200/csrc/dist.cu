@@ -228,6 +228,35 @@ int allreduce_u64(Comm* c, uint64_t* v, cudaStream_t s) {
   return ATOS_OK;
 }
 
+int allgather_host(Comm* c, const void* in, size_t bytes, void* out, cudaStream_t s) {
+  const int P = c->nranks;
+  if (c->h_a2a) {
+    std::vector<char> sbuf((size_t)P * bytes);
+    for (int p = 0; p < P; ++p) memcpy(sbuf.data() + (size_t)p * bytes, in, bytes);
+    std::vector<uint64_t> cnt(P, bytes);
+    if (c->h_a2a(c->h_user, sbuf.data(), cnt.data(), out, cnt.data()) != 0) {
+      set_error("host alltoallv (allgather) failed");
+      return ATOS_ERR_NCCL;
+    }
+    return ATOS_OK;
+  }
+  static thread_local DevBuf buf;
+  ATOS_TRY(buf.ensure((size_t)P * bytes * 2));
+  char* d_in = buf.as<char>();
+  char* d_out = d_in + (size_t)P * bytes;
+  ATOS_CUDA(cudaMemcpyAsync(d_in, in, bytes, cudaMemcpyHostToDevice, s));
+  NcclApi& api = nccl();
+  ATOS_NCCL(api.GroupStart());
+  for (int p = 0; p < P; ++p) {
+    ATOS_NCCL(api.Send(d_in, bytes, ncclUint8, p, (ncclComm_t)c->nccl, s));
+    ATOS_NCCL(api.Recv(d_out + (size_t)p * bytes, bytes, ncclUint8, p, (ncclComm_t)c->nccl, s));
+  }
+  ATOS_NCCL(api.GroupEnd());
+  ATOS_CUDA(cudaMemcpyAsync(out, d_out, (size_t)P * bytes, cudaMemcpyDeviceToHost, s));
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  return ATOS_OK;
+}
+
 int allreduce_f64(Comm* c, double* v, cudaStream_t s) {
   if (c->h_ar) {
     ATOS_CUDA(cudaStreamSynchronize(s));

@@ -67,6 +67,11 @@ struct Part {
   DevBuf ghost_a, ghost_b, touched, outbox, inbox, out_val, in_val, pack;
   DevBuf bsp_fa, bsp_fb, bsp_off, bsp_tmp, bsp_ctr;  // BSP baselines (bsp.cu)
   DevBuf nb_ring, nb_ctl, nb_peers;                   // barrier-free partitioned PageRank (nobarrier.cu)
+  // barrier-free across PROCESSES (nobarrier.cu run_nobarrier_mp): this rank's peer-visible block
+  // (cudaMalloc, exported with a CUDA IPC handle) and the peers' blocks mapped into this process
+  void* nb_ipc = nullptr;
+  size_t nb_ipc_bytes = 0;
+  std::vector<void*> nb_peer_base;
   uint64_t ring_cap = 0;
   void* host_pinned = nullptr;      // 4 KB pinned scratch for control-block reads
   bool ring_clean = false;          // every ring slot is EMPTY
@@ -96,6 +101,8 @@ struct ExchangeIO {
 int exchange_loopback(std::vector<ExchangeIO>& io, size_t val_bytes, cudaStream_t s);
 int exchange_nccl(Comm* c, ExchangeIO& io, size_t val_bytes, cudaStream_t s, uint64_t* bytes_sent);
 int allreduce_u64(Comm* c, uint64_t* v, cudaStream_t s);
+// every rank's `bytes` bytes (host memory) into out[rank * bytes] on every rank
+int allgather_host(Comm* c, const void* in, size_t bytes, void* out, cudaStream_t s);
 int allreduce_f64(Comm* c, double* v, cudaStream_t s);
 
 }  // namespace atos

@@ -235,6 +235,9 @@ int create_single(atos_csr* g, const int64_t* row_ptr, const int32_t* col, int w
   p.v_end = n;
   p.n_local = n;
   p.m_local = m;
+  // device input may still be in flight on the caller's stream (e.g. just produced by torch): the
+  // creation streams below are non-blocking, so wait for the device first
+  if (where == ATOS_MEM_DEVICE) ATOS_CUDA(cudaDeviceSynchronize());
   UploadCtx cx;
   ATOS_CUDA(cudaStreamCreateWithFlags(&cx.cs, cudaStreamNonBlocking));
   ATOS_CUDA(cudaStreamCreateWithFlags(&cx.ks, cudaStreamNonBlocking));

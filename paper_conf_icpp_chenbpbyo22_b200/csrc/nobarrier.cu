@@ -65,6 +65,8 @@ struct NbParams {
   double alpha, eps;
   unsigned long long watchdog_ns;
   unsigned long long timeout_ns;  // cfg.timeout_s as a device deadline from kernel start (0: none)
+  int self;                       // -1: loopback (this kernel serves every partition); else the only
+                                  // partition this process serves (one partition per process, peers mapped)
 };
 
 __device__ __forceinline__ unsigned long long nb_tag(unsigned long long idx, uint32_t item) {
@@ -103,9 +105,11 @@ __device__ __forceinline__ void nb_push(const NbParams& prm, bool act, uint32_t 
 
 }  // namespace
 
-// Rank / residue init of every partition (Alg.3, R-PR-init): rank = 1 - alpha, residue = 0.
+// Rank / residue init of every partition this process serves (Alg.3, R-PR-init): rank = 1 - alpha,
+// residue = 0.
 __global__ void k_nb_init_vertices(NbParams prm, double one_minus_alpha) {
-  for (uint32_t p = 0; p < prm.P; ++p) {
+  const uint32_t p0 = prm.self < 0 ? 0u : (uint32_t)prm.self, p1 = prm.self < 0 ? prm.P : p0 + 1;
+  for (uint32_t p = p0; p < p1; ++p) {
     const NbPeer pe = prm.peers[p];
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < pe.n_local;
          v += (int64_t)gridDim.x * blockDim.x) {
@@ -154,7 +158,7 @@ __global__ void __launch_bounds__(kNbBlock, ATOS_NB_MINB) k_nobarrier(NbParams p
   __shared__ int s_quit;
   __shared__ uint32_t s_off[kNbBlock], s_start[kNbBlock], s_wsum[kNbBlock / 32];
   __shared__ double s_delta[kNbBlock];
-  const uint32_t q = blockIdx.x % (prm.P * prm.S);
+  const uint32_t q = prm.self < 0 ? blockIdx.x % (prm.P * prm.S) : (uint32_t)prm.self * prm.S + blockIdx.x % prm.S;
   const uint32_t me = q / prm.S, sub0 = q % prm.S;
   const NbPeer self = prm.peers[me];
   __shared__ uint32_t s_sq;
@@ -333,7 +337,8 @@ __global__ void __launch_bounds__(kNbBlock, ATOS_NB_MINB) k_nobarrier(NbParams p
 // rank_out = rank / n_global (R-PR-4); residual sum into *sum.
 __global__ void k_nb_finalize(NbParams prm, double n_global, double* sum) {
   double acc = 0.0;
-  for (uint32_t p = 0; p < prm.P; ++p) {
+  const uint32_t p0 = prm.self < 0 ? 0u : (uint32_t)prm.self, p1 = prm.self < 0 ? prm.P : p0 + 1;
+  for (uint32_t p = p0; p < p1; ++p) {
     const NbPeer pe = prm.peers[p];
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < pe.n_local;
          v += (int64_t)gridDim.x * blockDim.x) {
@@ -361,22 +366,192 @@ __global__ void k_nb_bfs_seed(NbParams prm, uint32_t o, uint32_t l) {
   nb_push(prm, lane_id() == 0, o, l);
 }
 
+// ---------------------------------------------------------------- across processes
+// One partition per process (torchrun / the host transport).  Each rank keeps its peer-visible state in
+// ONE cudaMalloc block -- its S rings, their counters, its residue (PageRank) or depth words (BFS), its
+// in-queue bits, and a global word block -- exported once with a CUDA IPC handle; the handles are
+// all-gathered over the communicator and every peer block is mapped (cudaIpcOpenMemHandle, lazy peer
+// access: NVLink peer memory across GPUs, the same memory on one GPU).  The kernel is the loopback one:
+// this process's CTAs serve only its own sub-queues, and a remote relaxation is an atomic on the owner's
+// block plus, on activation, a push into the owner's ring.  Termination is the same global quiescence,
+// read over every rank's counters.  Host barriers (allreduce) separate the phases that write another
+// rank's memory: init -> (PageRank) init residues -> seeds -> kernels -> end (no rank frees or reuses its
+// block while a peer's kernel may still read its counters).
+struct NbLayout {
+  size_t ring, ctl, state, inq, glob, total;
+};
+static NbLayout nb_layout(int64_t n_local, uint32_t S) {
+  auto al = [](size_t x) { return (x + 255) / 256 * 256; };
+  NbLayout L;
+  const uint64_t cap = nb_pow2((uint64_t)std::max<int64_t>(n_local, 1024));
+  L.ring = 0;
+  L.ctl = al(L.ring + (size_t)S * cap * 8);
+  L.state = al(L.ctl + (size_t)S * sizeof(NbCtl));
+  L.inq = al(L.state + (size_t)std::max<int64_t>(n_local, 1) * 8);
+  L.glob = al(L.inq + ((size_t)n_local / 32 + 1) * 4);
+  L.total = al(L.glob + sizeof(NbGlob) + 8);
+  return L;
+}
+
+static int nb_barrier(atos_csr* g, cudaStream_t s) {
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  uint64_t z = 0;
+  return allreduce_u64(g->comm, &z, s);
+}
+
+static int run_nobarrier_mp(atos_csr* g, bool bfs, double alpha, double eps, double* rank_out, uint32_t* depth_out,
+                            int64_t src, const Resolved& r, atos_stats* st) {
+  cudaStream_t s = r.stream;
+  const uint32_t P = (uint32_t)g->nranks, me = (uint32_t)g->rank;
+  if (P > kNbMaxParts) {
+    set_error("barrier_free: at most %u ranks (got %u)", kNbMaxParts, P);
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  if (!bfs && r.check_size > 0) {
+    set_error("barrier_free: check_size sweeps are single-partition only");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  uint32_t S = bfs ? 4u : (P >= 4 ? 1u : 2u);
+  if (const char* e = getenv("ATOS_NB_SUBQ")) S = (uint32_t)std::max(1, std::min(16, atoi(e)));
+  const uint32_t B = (uint32_t)((g->n + P - 1) / P);
+  Part& p = g->parts[0];
+  std::vector<int64_t> nl(P);
+  for (uint32_t i = 0; i < P; ++i) {
+    int64_t b = 0, e = 0;
+    atos_partition_range(g->n, (int)P, (int)i, &b, &e);
+    nl[i] = e - b;
+  }
+  const NbLayout mine = nb_layout(nl[me], S);
+  // 1. the peer-visible block and the peers' mappings (once per handle)
+  if (!p.nb_ipc) {
+    ATOS_CUDA(cudaMalloc(&p.nb_ipc, mine.total));
+    p.nb_ipc_bytes = mine.total;
+    cudaIpcMemHandle_t h;
+    ATOS_CUDA(cudaIpcGetMemHandle(&h, p.nb_ipc));
+    std::vector<cudaIpcMemHandle_t> all(P);
+    ATOS_TRY(allgather_host(g->comm, &h, sizeof(h), all.data(), s));
+    p.nb_peer_base.assign(P, nullptr);
+    for (uint32_t i = 0; i < P; ++i) {
+      if (i == me) continue;
+      ATOS_CUDA(cudaIpcOpenMemHandle(&p.nb_peer_base[i], all[i], cudaIpcMemLazyEnablePeerAccess));
+    }
+  }
+  std::vector<NbPeer> peers(P);
+  for (uint32_t i = 0; i < P; ++i) {
+    char* b = i == me ? (char*)p.nb_ipc : (char*)p.nb_peer_base[i];
+    const NbLayout L = nb_layout(nl[i], S);
+    const uint64_t cap = nb_pow2((uint64_t)std::max<int64_t>(nl[i], 1024));
+    peers[i] = NbPeer{i == me ? p.row_ptr : nullptr, i == me ? p.col : nullptr,
+                      (!bfs && i == me) ? rank_out : nullptr, bfs ? nullptr : (double*)(b + L.state),
+                      (unsigned long long*)(b + L.ring), (NbCtl*)(b + L.ctl), cap - 1, (uint32_t)nl[i], 0,
+                      bfs ? (uint32_t*)(b + L.state) : nullptr, (uint32_t*)(b + L.inq)};
+  }
+  const size_t tbl = sizeof(NbPeer) * P;
+  ATOS_TRY(p.nb_peers.ensure(tbl));
+  ATOS_CUDA(cudaMemcpyAsync(p.nb_peers.p, peers.data(), tbl, cudaMemcpyHostToDevice, s));
+  char* own = (char*)p.nb_ipc;
+  NbGlob* glob = (NbGlob*)((char*)(me == 0 ? p.nb_ipc : p.nb_peer_base[0]) + nb_layout(nl[0], S).glob);
+  double* sum = (double*)(own + mine.glob + sizeof(NbGlob));
+  int shift = -1;
+  if ((B & (B - 1)) == 0) {
+    shift = 0;
+    while ((1u << shift) < B) ++shift;
+  }
+  NbParams prm{(const NbPeer*)p.nb_peers.p, glob, P, B, shift, S, alpha, eps, r.watchdog_ns,
+                r.timeout_s > 0 ? (unsigned long long)(r.timeout_s * 1e9) : 0ull, (int)me};
+  const int gs = 148 * 8;
+  // 2. own state (rings, counters, global words, residue / depth, in-queue bits), then a barrier
+  ATOS_CUDA(cudaMemsetAsync(own + mine.ring, 0, mine.state - mine.ring, s));
+  ATOS_CUDA(cudaMemsetAsync(own + mine.inq, 0, mine.total - mine.inq, s));
+  if (bfs) {
+    ATOS_CUDA(cudaMemsetAsync(own + mine.state, 0xFF, (size_t)std::max<int64_t>(nl[me], 1) * 4, s));
+  } else {
+    k_nb_init_vertices<<<gs, 256, 0, s>>>(prm, 1.0 - alpha);
+    ++g_launches;
+  }
+  ATOS_CUDA(cudaGetLastError());
+  ATOS_TRY(nb_barrier(g, s));
+  // 3. PageRank: every rank's rows add their initial mass into the owners' residues; then a barrier
+  if (!bfs) {
+    if (nl[me]) {
+      k_nb_init_edges<<<gs, 256, 0, s>>>(prm, me, (1.0 - alpha) * alpha);
+      ++g_launches;
+    }
+    ATOS_TRY(nb_barrier(g, s));
+  }
+  // 4. seeds (own ring), then a barrier: no kernel may observe quiescence before every seed is queued
+  if (bfs) {
+    if (src >= (int64_t)me * B && src < (int64_t)me * B + nl[me]) {
+      k_nb_bfs_seed<<<1, 32, 0, s>>>(prm, me, (uint32_t)(src - (int64_t)me * B));
+      ++g_launches;
+    }
+  } else if (nl[me]) {
+    k_nb_seed<<<gs, 256, 0, s>>>(prm, me);
+    ++g_launches;
+  }
+  ATOS_CUDA(cudaGetLastError());
+  ATOS_TRY(nb_barrier(g, s));
+  // 5. the persistent kernel of this rank
+  int grid = 0;
+  const void* fn = bfs ? (const void*)k_nobarrier<true> : (const void*)k_nobarrier<false>;
+  ATOS_TRY(persistent_grid(fn, kNbBlock, 0, &grid));
+  if (r.num_blocks > 0) grid = std::min(grid, r.num_blocks);
+  grid = std::max<int>((int)S, grid - grid % (int)S);
+  WorkerTimer wt;
+  wt.start(s);
+  void* args[] = {(void*)&prm};
+  ATOS_CUDA(cudaLaunchCooperativeKernel(fn, grid, kNbBlock, args, 0, s));
+  ++g_launches;
+  wt.stop(s);
+  if (stream_wait(s, r.timeout_s) == ATOS_ERR_TIMEOUT) ATOS_CUDA(cudaStreamSynchronize(s));
+  // 6. every kernel has stopped before anyone reads results or reuses its block
+  ATOS_TRY(nb_barrier(g, s));
+  NbGlob hg{};
+  ATOS_CUDA(cudaMemcpy(&hg, glob, sizeof(NbGlob), cudaMemcpyDeviceToHost));
+  if (hg.abort) {
+    set_error("barrier_free %s: %s", bfs ? "BFS" : "PageRank",
+              hg.abort == 2 ? "timeout_s exceeded" : "no progress (watchdog)");
+    return ATOS_ERR_TIMEOUT;
+  }
+  double hsum = 0.0;
+  if (bfs) {
+    if (nl[me]) ATOS_CUDA(cudaMemcpyAsync(depth_out, own + mine.state, (size_t)nl[me] * 4, cudaMemcpyDeviceToDevice, s));
+  } else {
+    ATOS_CUDA(cudaMemsetAsync(sum, 0, 8, s));
+    k_nb_finalize<<<gs, 256, 0, s>>>(prm, (double)g->n, sum);
+    ++g_launches;
+    ATOS_CUDA(cudaMemcpyAsync(&hsum, sum, 8, cudaMemcpyDeviceToHost, s));
+  }
+  ATOS_CUDA(cudaStreamSynchronize(s));
+  if (!bfs) ATOS_TRY(allreduce_f64(g->comm, &hsum, s));
+  if (st) {
+    std::vector<NbCtl> hc(S);
+    ATOS_CUDA(cudaMemcpy(hc.data(), own + mine.ctl, S * sizeof(NbCtl), cudaMemcpyDeviceToHost));
+    for (uint32_t j = 0; j < S; ++j) {
+      st->pops += hc[j].done;
+      st->pushes += hc[j].tail;
+    }
+    st->edges += hg.edges;  // every rank's edge visits (the counter is global)
+    st->rounds += 1;
+    if (!bfs) st->residual_sum = hsum;
+    st->worker_ms += wt.elapsed();
+  }
+  return ATOS_OK;
+}
+
 // Shared driver: PageRank (rank_out) or BFS (depth_out, src).
 static int run_nobarrier(atos_csr* g, bool bfs, double alpha, double eps, double* rank_out, uint32_t* depth_out,
                          int64_t src, const Resolved& r, atos_stats* st) {
   cudaStream_t s = r.stream;
-  if (g->comm) {
-    set_error("barrier_free: only loopback partitions (num_parts > 1 on one device) in this build");
-    return ATOS_ERR_UNSUPPORTED;
-  }
-  const uint32_t P = (uint32_t)g->num_parts;
-  if (P < 2 || P > kNbMaxParts) {
-    set_error("barrier_free: needs a loopback-partitioned graph with 2..%u partitions (got %u)", kNbMaxParts, P);
-    return ATOS_ERR_UNSUPPORTED;
-  }
   if (r.knobs_set) {
     set_error("barrier_free: persistent=0, dedupe=0, worker, fetch_size, queue_capacity, depth_state and "
               "engine_variant do not apply to the barrier-free kernel (its worker is fixed, DESIGN.md section 7)");
+    return ATOS_ERR_UNSUPPORTED;
+  }
+  if (g->comm) return run_nobarrier_mp(g, bfs, alpha, eps, rank_out, depth_out, src, r, st);
+  const uint32_t P = (uint32_t)g->num_parts;
+  if (P < 2 || P > kNbMaxParts) {
+    set_error("barrier_free: needs a loopback-partitioned graph with 2..%u partitions (got %u)", kNbMaxParts, P);
     return ATOS_ERR_UNSUPPORTED;
   }
   if (!bfs && r.check_size > 0) {
@@ -429,7 +604,7 @@ static int run_nobarrier(atos_csr* g, bool bfs, double alpha, double eps, double
     while ((1u << shift) < B) ++shift;
   }
   NbParams prm{(const NbPeer*)base, glob, P, B, shift, S, alpha, eps, r.watchdog_ns,
-                r.timeout_s > 0 ? (unsigned long long)(r.timeout_s * 1e9) : 0ull};
+                r.timeout_s > 0 ? (unsigned long long)(r.timeout_s * 1e9) : 0ull, -1};
   const int gs = 148 * 8;
   if (bfs) {
     const uint32_t o = (uint32_t)(src / B);

@@ -63,6 +63,18 @@ def _worker(rank, world, port, scale, q):
         iso = int(np.sum(np.diff(rp) == 0))
         # stats.residual_sum of a distributed call is already the sum over ranks (allreduce in the library)
         assert abs(tot[0].item() + st["residual_sum"] / 0.15 - (full.n - 0.85 * iso)) < 1e-9 * full.n
+        # NEXT-4 across processes: the barrier-free kernel with every peer's rings / state mapped through CUDA
+        # IPC (the ranks' kernels time-share the one GPU here); bit-exact BFS, in-tolerance PageRank
+        for s in (gen.pick_source(full, 1), 0):
+            d, st = atos.bfs(csr, s, barrier_free=1, timeout_s=120)
+            np.testing.assert_array_equal(d.cpu().numpy().view(np.uint32), oracle.bfs(rp, ci, s)[vb:ve])
+        r, st = atos.pagerank(csr, 0.85, 1e-6, barrier_free=1, timeout_s=120)
+        x = r.cpu().numpy()
+        assert (np.abs(x - ref[vb:ve]) / np.maximum(ref[vb:ve], 1e-300)).max() <= 1e-4
+        assert np.all(x <= ref[vb:ve] * (1 + 1e-9) + 1e-15)
+        tot = torch.tensor([x.sum() * full.n], dtype=torch.float64)
+        dist.all_reduce(tot)
+        assert abs(tot[0].item() + st["residual_sum"] / 0.15 - (full.n - 0.85 * iso)) < 1e-9 * full.n
         csr.close()
         comm.close()
         q.put((rank, "ok"))
