@@ -173,11 +173,7 @@ constexpr uint32_t kGoBig = 0xFFFFFFFFu;
 // slower (its hub spans are already one coalesced load per lane) -- the launcher picks it per graph.
 constexpr uint32_t kPfKU = 4;                              // buffer sized for up to 4 edges per lane
 constexpr uint32_t kPfWarpBytes = 2u * 32u * kPfKU * 6u;   // 2 stages x (u32 id + u16 owner) per edge slot
-#ifdef ATOS_PF_HUB
-constexpr bool kPfHubBuild = true;
-#else
-constexpr bool kPfHubBuild = false;
-#endif
+
 __device__ __forceinline__ void cp_async4(void* smem, const void* gmem, unsigned long long pol) {
   const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
   asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(sa), "l"(gmem), "l"(pol)
@@ -851,37 +847,7 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
         asm volatile("cp.async.wait_all;" ::: "memory");
         __syncwarp();
       } else {
-#ifdef ATOS_PF_HUB
-      // hub-span prefetch: when the NEXT iteration's warp span lies in one row (the fast path below), its 32*KU
-      // contiguous ids are staged with cp.async into a per-warp double buffer while this iteration runs
-      uint32_t* hb = (uint32_t*)((unsigned char*)(cown + kCown) + (size_t)warp_id() * kPfWarpBytes);
-      auto hub_span = [&](uint32_t b0, uint32_t buf) {
-        const uint32_t wf = b0 + (r & ~31u) * KU;
-        if (table && wf < total) {
-          const uint32_t c = wf / wspan;
-          const uint32_t lo = cown[c], hi = c + 1 < nchunk ? cown[c + 1] : nready - 1;
-          if (lo == hi) {
-            const uint32_t st0 = s.start[lo] + (wf - s.off[lo]), len = min(wf + wspan, total) - wf;
-#pragma unroll
-            for (int k = 0; k < KU; ++k)
-              if (k * 32 + lane_id() < len)
-                cp_async4(hb + buf * 32 * kPfKU + k * 32 + lane_id(), app.col + st0 + k * 32 + lane_id(),
-                          app.pol_first);
-          }
-        }
-        cp_async_commit();
-      };
-      hub_span(0, 0);
-      uint32_t hbuf = 0;
-#endif
       for (uint32_t base = 0; base < total; base += G * KU) {
-#ifdef ATOS_PF_HUB
-        hub_span(base + G * KU, hbuf ^ 1u);
-        cp_async_wait1();
-        __syncwarp();
-        const uint32_t hcur = hbuf;
-        hbuf ^= 1u;
-#endif
         const uint32_t wfirst = base + (r & ~31u) * KU;
         if (wfirst >= total) continue;  // warp-uniform; no collective below is skipped by part of a warp
         const uint32_t wlast = min(wfirst + wspan, total) - 1;
@@ -909,13 +875,6 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
           const uint32_t st0 = s.start[olo] + (wfirst - s.off[olo]);
           const uint32_t len = wlast - wfirst + 1;
           const Payload p = s.pay[olo];
-#ifdef ATOS_PF_HUB
-          if (table) {
-#pragma unroll
-            for (int k = 0; k < KU; ++k)
-              if (k * 32 + lane_id() < len) w[k] = hb[hcur * 32 * kPfKU + k * 32 + lane_id()];
-          } else
-#endif
 #pragma unroll
           for (int k = 0; k < KU; ++k)
             if (k * 32 + lane_id() < len) {
@@ -992,10 +951,6 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
         }
         pusher.push_n<KU>(q, want, out, P.watchdog_ns);
       }
-#ifdef ATOS_PF_HUB
-      asm volatile("cp.async.wait_all;" ::: "memory");
-      __syncwarp();
-#endif
       }  // !PF
     } else if (MODE == MODE_WARP) {
       for (uint32_t k = 0; k < nready; ++k) {
@@ -1076,7 +1031,7 @@ inline size_t relax_worker_smem(int mode, uint32_t block, uint32_t fetch, bool p
   uint32_t K = mode == MODE_THREAD ? 32u * fetch : fetch;
   uint32_t groups = mode == MODE_CTA ? 1u : nwarps;
   return (size_t)nwarps * kPushBuf * 4 + group_smem_bytes<Payload>(K) * groups +
-         (mode == MODE_CTA ? kCown * 4 + (pf || kPfHubBuild ? (size_t)nwarps * kPfWarpBytes : 0) : 0);
+         (mode == MODE_CTA ? kCown * 4 + (pf ? (size_t)nwarps * kPfWarpBytes : 0) : 0);
 }
 
 }  // namespace atos

@@ -191,6 +191,12 @@ __global__ void k_pr_sweep(const double* res, int64_t n, double eps, Ring q, uin
 #define ATOS_PF_LOWDEG 1
 #endif
 constexpr bool kPfLowDegree = ATOS_PF_LOWDEG != 0;
+#ifndef ATOS_HD_KU
+#define ATOS_HD_KU 4    // high-degree graphs: edges in flight per thread of the (256, MINB) build
+#endif
+#ifndef ATOS_HD_MINB
+#define ATOS_HD_MINB 5  // resident 256-thread CTAs per SM the register budget is sized for
+#endif
 
 static inline uint64_t pow2_at_least(uint64_t x) {
   uint64_t c = 1;
@@ -328,7 +334,7 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
     if (block == 256 && r.persistent && r.engine_variant != 1) {
       const bool low_degree = p.n_local > 0 && p.m_local < 8 * p.n_local;
       if (low_degree) return launch_relax_mode<App, MODE_CTA, 2, 5, kPfLowDegree>(app, P, r, block, p, st);
-      return launch_relax_mode<App, MODE_CTA, 4, 5>(app, P, r, block, p, st);
+      return launch_relax_mode<App, MODE_CTA, ATOS_HD_KU, ATOS_HD_MINB>(app, P, r, block, p, st);
     }
     if (App::kPfCta && r.persistent && r.engine_variant != 1)
       return launch_relax_mode<App, MODE_CTA, kU, ATOS_MINB, true>(app, P, r, block, p, st);

@@ -139,3 +139,19 @@ def test_c5_pagerank_residual_certificate(c5):
     assert abs(x.sum() + st["residual_sum"] / (1 - alpha) - (n - alpha * iso)) < 1e-9 * n
     # and the library's residual sum agrees with the certificate's
     assert abs(st["residual_sum"] - res.sum()) < 1e-6 * n
+
+
+@pytest.mark.parametrize("P", [2, 8])
+def test_c5_partitioned_bfs_vs_oracle(c5, P):
+    """The bench's partitioned C5 lines (exchange rounds and barrier-free over P loopback partitions) against
+    the ORACLE, not only against the single-partition result."""
+    csr, rp, ci, n, sources = c5
+    src = sources[0]
+    want = oracle.bfs(rp, ci, src)
+    pc = atos.CSR(torch.from_numpy(rp), torch.from_numpy(ci), num_parts=P)
+    out = torch.empty(n, dtype=torch.int32, device=DEV)
+    d, st = atos.bfs(pc, src, out=out)
+    np.testing.assert_array_equal(as_u32(d), want)
+    d, st = atos.bfs(pc, src, out=out, barrier_free=1)
+    np.testing.assert_array_equal(as_u32(d), want)
+    pc.close()
