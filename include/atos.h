@@ -86,7 +86,8 @@ typedef struct {
     double   worker_ms;         /* device time of the worker kernel(s) alone (persistent launch, or the sum
                                    of the discrete launches incl. their host round trips), CUDA events */
     uint64_t timeline_len;      /* samples written to cfg->timeline */
-    uint64_t flags;             /* bit 0: BFS re-ran with the u32 depth state (depth >= 126 met) */
+    uint64_t flags;             /* bit 0: BFS re-ran with the u32 depth state (depth >= 126 met); bit 1: BFS started
+                                   with the u32 state because an earlier call on this graph met depth >= 126 */
     uint64_t max_queue_occupancy; /* largest number of published-but-unclaimed items (tail - head) any worker
                                    saw at a claim (persistent runs; discrete: the largest frontier) */
 } atos_stats;
@@ -96,8 +97,9 @@ typedef struct {
     int      persistent;        /* 1 persistent kernel (default), 0 discrete per-frontier launches */
     int      worker;            /* 1 thread, 32 warp, 64..1024 CTA; 0 = per-app default (CTA: BFS 256, PageRank 512,
                                    colouring 1024) */
-    int      fetch_size;        /* items per pop per worker (FETCH_SIZE); 0 = default (CTA: worker size,
-                                   colouring min(worker,128); warp 8; thread 1) */
+    int      fetch_size;        /* items per pop per worker (FETCH_SIZE); 0 = default (CTA: worker size
+                                   for BFS, min(worker,256) for PageRank, min(worker,128) for colouring; warp 8;
+                                   thread 1) */
     int      num_blocks;        /* 0 = occupancy max (persistent) / proportional to the frontier (discrete) */
     int      block_threads;     /* threads per block for thread/warp workers; 0 = 256 */
     int      dedupe;            /* 1 (default): in-queue bitmap, a vertex is queued at most once at a time;
@@ -115,7 +117,9 @@ typedef struct {
     double   timeout_s;         /* 0 = none; else the call fails with ATOS_ERR_TIMEOUT */
     void*    stream;            /* cudaStream_t; NULL = legacy default stream */
     atos_stats* stats;          /* optional out */
-    int      l2_persist;        /* 1: L2 persisting access-policy window on queue counters + hot state */
+    int      l2_persist;        /* 1: L2 persisting access-policy window on the hot per-vertex state (BFS state
+                                   bytes / depth words, PageRank residue).  The queue counters always carry
+                                   per-access L2 evict_last hints (createpolicy), independent of this knob */
     int      big_threshold;     /* persistent CTA/warp workers: a popped vertex with more edges than this is
                                    split into chunks any worker may claim (hub assist); 0 = auto, <0 = off */
     int      big_chunk;         /* edges per hub-assist chunk; 0 = auto */

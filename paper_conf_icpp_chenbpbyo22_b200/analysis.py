@@ -29,8 +29,10 @@ def overwork_factor(app: str, pops: int, bsp_pops: int | None = None, n: int | N
 def throughput_series(table) -> tuple[np.ndarray, np.ndarray]:
     """(t_us at interval mid-points, tasks completed per microsecond) from a timeline table
     (rows: globaltimer ns since the first sample, done, tail, head -- see timeline_table())."""
-    t = np.asarray(table[:, 0], dtype=np.float64) / 1e3
-    done = np.asarray(table[:, 1], dtype=np.float64)
+    tab = np.asarray(table, dtype=np.float64)
+    tab = tab[np.argsort(tab[:, 0], kind="stable")]  # samplers of adjacent intervals can land out of order
+    t = tab[:, 0] / 1e3
+    done = tab[:, 1]
     if t.size < 2:
         return np.zeros(0), np.zeros(0)
     dt = np.diff(t)

@@ -202,8 +202,11 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
     return ATOS_ERR_INVALID_ARG;
   }
   r->fetch = d.fetch_size;
+  // CTA defaults: BFS fetch = worker; colouring min(worker, 128); PageRank min(worker, 256) (512:256 vs
+  // 512:512 measured C3 61.7 vs 63.6 ms, C5 even -- profiles/r02_pr_fetch_sweep.txt)
   if (r->fetch == 0)
-    r->fetch = (r->worker >= 64) ? (app == 'c' ? std::min(r->worker, 128) : r->worker) : (r->worker == 32 ? 8 : 1);
+    r->fetch = (r->worker >= 64) ? (app == 'c' ? std::min(r->worker, 128) : (app == 'p' ? std::min(r->worker, 256) : r->worker))
+                                 : (r->worker == 32 ? 8 : 1);
   if (r->fetch < 1 || r->fetch > 4096) {
     set_error("fetch_size must be in [1, 4096] (got %d)", r->fetch);
     return ATOS_ERR_INVALID_ARG;

@@ -26,6 +26,9 @@ namespace atos {
 //     At termination every queued vertex was popped, so all INQ bits are 0.
 //   * two-phase relax (pre: prefilter load, post: decision + atomics) so the
 //     engine can keep several edges' loads in flight per thread.
+#ifndef ATOS_FUSED_BEGIN
+#define ATOS_FUSED_BEGIN 1
+#endif
 constexpr uint32_t kInq = 0x80000000u;
 constexpr uint32_t kDepthMask = 0x7FFFFFFFu;
 
@@ -59,7 +62,9 @@ template <bool PART, bool ACQ = true>
 struct BfsAppT {
   static constexpr bool kAcquirePop = ACQ;
   static constexpr bool kPfCta = false;  // CTA workers other than the (256,5) build: direct col loads
-  static constexpr bool kFusedBegin = false;
+  // fused consume + begin (engine.cuh consume_slot_fused): begin() only clears the queued flag / reads the
+  // depth, so a speculative begin on a slot lost to a lapping producer can at worst cause a duplicate push
+  static constexpr bool kFusedBegin = ATOS_FUSED_BEGIN != 0 && !PART;
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
   const uint32_t* __restrict__ row_ptr;
@@ -173,9 +178,6 @@ struct BfsByteAppT {
   // ordering through the address dependency alone); the AND itself can then stay relaxed.
   static constexpr bool kAcquirePop = true;
   static constexpr bool kPfCta = false;
-#ifndef ATOS_FUSED_BEGIN
-#define ATOS_FUSED_BEGIN 1
-#endif
   static constexpr bool kFusedBegin = ATOS_FUSED_BEGIN != 0 && !PART;  // consume_slot_fused (engine.cuh)
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // the 32-bit word holding w's state byte (prefilter and CAS guess)

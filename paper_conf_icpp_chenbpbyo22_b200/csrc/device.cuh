@@ -166,6 +166,38 @@ __device__ __forceinline__ void st_u8_hint(uint8_t* a, uint32_t v, unsigned long
   asm volatile("st.global.L2::cache_hint.u8 [%0], %1, %2;" ::"l"(a), "h"((uint16_t)v), "l"(pol) : "memory");
 }
 
+// Queue counters (head / tail / done): every access carries an L2 evict_last cache-policy hint (the
+// north_star's "L2 persistence hints on the queue counters"), so the few hot counter lines are the last
+// candidates for eviction while the col stream (evict_first) and the state gathers churn through L2.
+// (The stream's access-policy window -- cfg.l2_persist -- is spent on the per-vertex state instead.)
+__device__ __forceinline__ unsigned long long ctr_policy() {
+  unsigned long long p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ unsigned long long ctr_ld(const unsigned long long* a) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(a), "l"(ctr_policy()) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ctr_add(unsigned long long* a, unsigned long long x) {
+  unsigned long long old;
+  asm volatile("atom.relaxed.gpu.global.add.L2::cache_hint.u64 %0, [%1], %2, %3;"
+               : "=l"(old) : "l"(a), "l"(x), "l"(ctr_policy()) : "memory");
+  return old;
+}
+__device__ __forceinline__ void ctr_red_release(unsigned long long* a, unsigned long long x) {
+  asm volatile("red.release.gpu.global.add.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(a), "l"(x), "l"(ctr_policy())
+               : "memory");
+}
+__device__ __forceinline__ unsigned long long ctr_read_acquire(unsigned long long* a) {
+  // an RMW returns the latest value in the location's coherence order
+  unsigned long long old;
+  asm volatile("atom.acquire.gpu.global.or.L2::cache_hint.b64 %0, [%1], 0, %2;"
+               : "=l"(old) : "l"(a), "l"(ctr_policy()) : "memory");
+  return old;
+}
+
 __device__ __forceinline__ void fence_sc_gpu() { asm volatile("fence.sc.gpu;" ::: "memory"); }
 __device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 
@@ -276,7 +308,7 @@ struct WarpPusher {
   __device__ __forceinline__ void publish(const Ring& q, uint32_t k, unsigned long long watchdog_ns) {
     // k <= 32 entries at buf[head .. head+k)
     unsigned long long base = 0;
-    if (lane_id() == 0) base = atomicAdd(&q.ctl->tail.v, (unsigned long long)k);
+    if (lane_id() == 0) base = ctr_add(&q.ctl->tail.v, (unsigned long long)k);
     base = __shfl_sync(0xffffffffu, base, 0);
     if (lane_id() < k) publish_one(q, base + lane_id(), buf[(head + lane_id()) & (kPushBuf - 1)], watchdog_ns);
     head = (head + k) & (kPushBuf - 1);

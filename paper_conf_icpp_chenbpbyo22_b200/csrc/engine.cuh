@@ -479,8 +479,8 @@ struct Worker {
           // number of workers (a high-diameter frontier) -- the fair share
           // visible / workers, at least kMinClaim, so one worker does not
           // serialise a whole small frontier while the others idle.
-          unsigned long long h = ld_relaxed(&q.ctl->head.v);
-          const unsigned long long t = ld_relaxed(&q.ctl->tail.v);
+          unsigned long long h = ctr_ld(&q.ctl->head.v);
+          const unsigned long long t = ctr_ld(&q.ctl->tail.v);
           if (h < t) {
             if (t - h > maxocc) maxocc = t - h;
             const unsigned long long nworkers =
@@ -489,7 +489,7 @@ struct Worker {
             const unsigned long long lo = K < kMinClaim ? K : kMinClaim;
             want = want < lo ? lo : (want > K ? K : want);
             if (t - h >= 2ull * want) {
-              const unsigned long long b = atomicAdd(&q.ctl->head.v, want);
+              const unsigned long long b = ctr_add(&q.ctl->head.v, want);
               *(unsigned long long*)&s.ctr[6] = b;
               s.ctr[4] = (uint32_t)want;
             } else {
@@ -539,8 +539,8 @@ struct Worker {
       // ------------------------------------------------------ 3. idle (f2)
       if (r == 0) {
         s.ctr[1] = npn;
-        const unsigned long long d = atom_read(&q.ctl->done.v);
-        const unsigned long long t = atom_read(&q.ctl->tail.v);
+        const unsigned long long d = ctr_read_acquire(&q.ctl->done.v);
+        const unsigned long long t = ctr_read_acquire(&q.ctl->tail.v);
         const uint32_t st = *(volatile uint32_t*)&q.ctl->status.v;
         if (d == t || st != 0) {
           if (PERSIST && d == t) tl_final(P);
@@ -582,8 +582,7 @@ struct Worker {
     if (PERSIST && r == 0 && nready) {
       // release reduction, no return value to wait for: the barrier above orders every warp's pushes
       // before the leader's release (cumulative), and nobody needs the old count (C5 BFS -1 %)
-      asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(&P.q.ctl->done.v), "l"((unsigned long long)nready)
-                   : "memory");
+      ctr_red_release(&P.q.ctl->done.v, (unsigned long long)nready);
     }
     if (r == 0) tl_sample(P);
     group_sync<MODE>();

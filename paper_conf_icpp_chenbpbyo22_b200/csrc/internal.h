@@ -116,6 +116,7 @@ struct atos_csr {
   int rank = 0, nranks = 1;
   int64_t max_degree = 0;
   bool symmetric_checked = false, symmetric = false;
+  bool bfs_deep_seen = false;              // a byte-state BFS on this graph met depth >= 126: start with u32 words
   bool relabeled = false;                  // degree layout (layout.cu): internal id = o2n[caller id]
   atos::DevBuf o2n, n2o, perm_out;         // u32[n] maps; output staging for host outputs
   std::mutex mu;

@@ -400,10 +400,15 @@ int bfs_single(atos_csr* g, Part& p, int64_t src, uint32_t* depth, const Resolve
   ATOS_TRY(ensure_queue(p, pow2_at_least(want), s));
   trace_mark("bfs: ensure_queue", true);
   // byte state first (dedupe mode); a traversal deeper than 125 levels re-runs with u32 words
-  if (r.dedupe && r.depth_state != 2) {
+  // A graph on which a byte-state traversal already ran out of depth codes (a high-diameter mesh or road
+  // network) starts every later BFS with the u32 words instead of paying the aborted first attempt again
+  // (stats.flags bit 1).
+  if (r.dedupe && r.depth_state != 2 && g->bfs_deep_seen && st) st->flags |= 2;
+  if (r.dedupe && r.depth_state != 2 && !g->bfs_deep_seen) {
     bool deep = false;
     ATOS_TRY(bfs_single_bytes(p, src, depth, r, st, &deep));
     if (!deep) return ATOS_OK;
+    g->bfs_deep_seen = true;
     if (st) {
       st->flags |= 1;  // re-run with the u32 state; rounds describe the final run (worker_ms keeps both)
       st->rounds = 0;

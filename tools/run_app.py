@@ -17,10 +17,16 @@ def main():
     seed = int(args.pop("seed", {"bfs": 5, "pr": 3, "gc": 4}[app]))
     reps = int(args.pop("reps", 1))
     tl = int(args.pop("timeline", 0))
-    knobs = {k: int(v) for k, v in args.items()}
-    g = gen.rmat(scale, ef, seed, device="cuda")
-    csr = atos.CSR.from_graph(g)
-    src = gen.pick_source(g, 105)
+    knobs = {k: int(v) for k, v in args.items() if k not in ("mesh", "keep")}
+    mesh = int(args.pop("mesh", 0))
+    if mesh:
+        g = gen.mesh(mesh, mesh, float(args.pop("keep", 1.0)), 2, device="cuda")
+        csr = atos.CSR.from_graph(g)
+        src = gen.mesh_centre_source(g, mesh, mesh)
+    else:
+        g = gen.rmat(scale, ef, seed, device="cuda")
+        csr = atos.CSR.from_graph(g)
+        src = gen.pick_source(g, 105)
     if args.pop("free_graph", None) or True:
         # keep only what the solver needs on the device (smaller ncu replay backups)
         stats = g.stats()
