@@ -103,6 +103,14 @@ def test_nccl_single_rank_communicator(rmat13):
     np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, s))
     r, st = atos.pagerank(part, 0.85, 1e-6)
     check_pr(rp, ci, r, st, 1e-6)
+    # the cross-process barrier-free path over NCCL (IPC handle all-gather by grouped send/recv)
+    d, st = atos.bfs(part, s, barrier_free=1)
+    np.testing.assert_array_equal(as_u32(d), oracle.bfs(rp, ci, s))
+    r, st = atos.pagerank(part, 0.85, 1e-6, barrier_free=1)
+    check_pr(rp, ci, r, st, 1e-6)
+    # atos_comm_gather over NCCL: the (only) slice lands on rank 0
+    full = comm.gather(g.n, d)
+    np.testing.assert_array_equal(as_u32(full), oracle.bfs(rp, ci, s))
     with pytest.raises(RuntimeError, match="INVALID_ARG"):
         comm.partition(g.n, 0, g.n - 1, g.row_ptr[:-1].to(DEV), g.col.to(DEV))
     part.close()
