@@ -5,6 +5,7 @@
 #include <atomic>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -159,6 +160,12 @@ struct Resolved {
   void* map_out = nullptr;
   bool* map_done = nullptr;
 };
+// smallest fair-share claim for an app's workers (EngineParams::min_claim): ATOS_MIN_CLAIM overrides `dflt`
+inline uint32_t min_claim_for(uint32_t dflt) {
+  const char* e = getenv("ATOS_MIN_CLAIM");
+  const long v = e ? atol(e) : 0;
+  return v > 0 ? (uint32_t)v : dflt;
+}
 // defaults: app = 'b' (bfs) / 'p' (pagerank) / 'c' (color)
 int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r);
 

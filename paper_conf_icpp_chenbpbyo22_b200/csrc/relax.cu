@@ -303,6 +303,7 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
   P.fetch = (uint32_t)r.fetch;
   P.watchdog_ns = r.watchdog_ns;
   P.h0 = P.t0 = 0;
+  P.min_claim = min_claim_for(kMinClaim);
   const int mode = mode_of(r.worker);
   const int block = mode == MODE_CTA ? r.worker : r.block_threads;
   // hub assist (persistent CTA / warp workers): auto threshold = 32 edges per
