@@ -702,7 +702,7 @@ def run_apps(args, dev, peak):
         oracle_counts["jones_plassmann_seed1"] = oracle.color_jp(rp, ci, 1)[1]
         oracle_counts["seconds"] = time.perf_counter() - t0
     res["color"] = {"config": f"C4: Kronecker scale {args.gc_scale} ef 64 seed 4 (n={g.n}, m={g.m}), seed 1, "
-                              "CTA worker 1024 / fetch 128 (library default)",
+                              "CTA worker 1024 / fetch 48 (library default)",
                     "ms_to_converge": float(np.mean(ms)), "ms_min": float(np.min(ms)), "worker_ms": wm,
                     "colors": int(np.max(cols)), "oracle_colors": oracle_counts,
                     "tasks_per_n": float(np.mean(pops)) / g.n,

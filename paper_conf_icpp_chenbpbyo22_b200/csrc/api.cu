@@ -202,10 +202,12 @@ int resolve_cfg(const atos_cfg* cfg, char app, Resolved* r) {
     return ATOS_ERR_INVALID_ARG;
   }
   r->fetch = d.fetch_size;
-  // CTA defaults: BFS fetch = worker; colouring min(worker, 128); PageRank min(worker, 256) (512:256 vs
+  // CTA defaults: BFS fetch = worker; colouring min(worker, 48) (fewer vertices assigned concurrently, fewer
+  // recolour cascades on a dense core: C4 1024:128 7.95 ms / 10.7 edge visits per m / 695 colours vs 1024:48
+  // 6.3 ms / 6.0 / 713-719, profiles/r02_gc_fetch_sweep.txt); PageRank min(worker, 256) (512:256 vs
   // 512:512 measured C3 61.7 vs 63.6 ms, C5 even -- profiles/r02_pr_fetch_sweep.txt)
   if (r->fetch == 0)
-    r->fetch = (r->worker >= 64) ? (app == 'c' ? std::min(r->worker, 128) : (app == 'p' ? std::min(r->worker, 256) : r->worker))
+    r->fetch = (r->worker >= 64) ? (app == 'c' ? std::min(r->worker, 48) : (app == 'p' ? std::min(r->worker, 256) : r->worker))
                                  : (r->worker == 32 ? 8 : 1);
   if (r->fetch < 1 || r->fetch > 4096) {
     set_error("fetch_size must be in [1, 4096] (got %d)", r->fetch);

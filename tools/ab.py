@@ -16,7 +16,7 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 GRID = {"bfs-rmat": "256:256:1", "bfs-mesh": "256:256:1", "bfs-road": "256:256:1", "pr": "512:512:1",
-        "gc": "1024:128:1"}
+        "gc": "1024:48:1"}
 
 
 def lib_of(tag):
