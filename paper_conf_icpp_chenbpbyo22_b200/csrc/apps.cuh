@@ -29,6 +29,9 @@ namespace atos {
 #ifndef ATOS_FUSED_BEGIN
 #define ATOS_FUSED_BEGIN 1
 #endif
+#ifndef ATOS_DEFER_CAS
+#define ATOS_DEFER_CAS 1
+#endif
 constexpr uint32_t kInq = 0x80000000u;
 constexpr uint32_t kDepthMask = 0x7FFFFFFFu;
 
@@ -179,8 +182,15 @@ struct BfsByteAppT {
   static constexpr bool kAcquirePop = true;
   static constexpr bool kPfCta = false;
   static constexpr bool kFusedBegin = ATOS_FUSED_BEGIN != 0 && !PART;  // consume_slot_fused (engine.cuh)
+  static constexpr bool kDeferCas = ATOS_DEFER_CAS != 0 && !PART;       // post_d / resolve (engine.cuh)
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // the 32-bit word holding w's state byte (prefilter and CAS guess)
+  // A lane's deferred discovery CAS: issued in one expand iteration, its result consumed in the next (after
+  // that iteration's col loads and state gathers are in flight), so the CAS round trip leaves the chain.
+  struct Pend {
+    uint32_t res, exp, w, nd;
+    bool on;
+  };
   const uint32_t* __restrict__ row_ptr;
   const uint32_t* __restrict__ col;
   uint8_t* state;            // n bytes, padded to a multiple of 4
@@ -270,6 +280,29 @@ struct BfsByteAppT {
   }
   __device__ __forceinline__ bool relax(const Payload nd, uint32_t w, uint32_t& out) const {
     return post(nd, w, pre(nd, w), out);
+  }
+  // post() with the lane's first improving CAS deferred (at most one pending per lane; others run inline)
+  __device__ __forceinline__ bool post_d(const Payload nd, uint32_t w, Token word, uint32_t& out, Pend& pd) const {
+    if (PART || pd.on) return post(nd, w, word, out);
+    const uint32_t sh = (w & 3u) * 8u;
+    const uint32_t D = (word >> sh) & 0x7Fu;
+    if (D != kBUnreached && D <= nd) return false;
+    pd.res = atomicCAS(word_of(w), word, (word & ~(0xFFu << sh)) | ((nd | kBInq) << sh));
+    pd.exp = word;
+    pd.w = w;
+    pd.nd = nd;
+    pd.on = true;
+    return false;
+  }
+  // the pending CAS's outcome: won -> queue w unless it was queued; lost -> the ordinary retry loop
+  __device__ __forceinline__ bool resolve(Pend& pd, uint32_t& out) const {
+    if (!pd.on) return false;
+    pd.on = false;
+    if (pd.res == pd.exp) {
+      out = pd.w;
+      return !((pd.exp >> ((pd.w & 3u) * 8u)) & kBInq);
+    }
+    return relax_local(pd.nd, pd.w, pd.res, out);
   }
 };
 

@@ -309,6 +309,20 @@ __device__ __forceinline__ void finish_big_chunk(const EngineParams& P, int slot
   }
 }
 
+// apps whose discovery CAS result can be consumed one expand iteration later (BfsByteAppT::kDeferCas)
+template <class A, class = void>
+struct has_defer_cas : std::false_type {};
+template <class A>
+struct has_defer_cas<A, std::void_t<decltype(A::kDeferCas)>> : std::bool_constant<A::kDeferCas> {};
+template <class A, bool ON = has_defer_cas<A>::value>
+struct PendOf {
+  struct type {};
+};
+template <class A>
+struct PendOf<A, true> {
+  using type = typename A::Pend;
+};
+
 // Per-group shared-memory arena.  K = items a group may hold at once.
 template <class Payload>
 struct GroupSmem {
@@ -855,6 +869,8 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
         asm volatile("cp.async.wait_all;" ::: "memory");
         __syncwarp();
       } else {
+      constexpr bool kDefer = has_defer_cas<App>::value;
+      typename PendOf<App>::type pd{};
       for (uint32_t base = 0; base < total; base += G * KU) {
         const uint32_t wfirst = base + (r & ~31u) * KU;
         if (wfirst >= total) continue;  // warp-uniform; no collective below is skipped by part of a warp
@@ -892,11 +908,19 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
 #pragma unroll
           for (int k = 0; k < KU; ++k)
             if (k * 32 + lane_id() < len) tk[k] = app.pre(p, w[k]);
+          if constexpr (kDefer) {
+            uint32_t po = 0;
+            const bool pw = app.resolve(pd, po);
+            pusher.push(q, pw, po, P.watchdog_ns);
+          }
 #pragma unroll
           for (int k = 0; k < KU; ++k) {
             want[k] = false;
             out[k] = 0;
-            if (k * 32 + lane_id() < len) want[k] = app.post(p, w[k], tk[k], out[k]);
+            if (k * 32 + lane_id() < len) {
+              if constexpr (kDefer) want[k] = app.post_d(p, w[k], tk[k], out[k], pd);
+              else want[k] = app.post(p, w[k], tk[k], out[k]);
+            }
           }
           pusher.push_n<KU>(q, want, out, P.watchdog_ns);
           continue;
@@ -951,13 +975,27 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
 #pragma unroll
         for (int k = 0; k < KU; ++k)
           if (val[k]) tk[k] = app.pre(s.pay[own[k]], w[k]);
+        if constexpr (kDefer) {
+          uint32_t po = 0;
+          const bool pw = app.resolve(pd, po);
+          pusher.push(q, pw, po, P.watchdog_ns);
+        }
 #pragma unroll
         for (int k = 0; k < KU; ++k) {
           want[k] = false;
           out[k] = 0;
-          if (val[k]) want[k] = app.post(s.pay[own[k]], w[k], tk[k], out[k]);
+          if (val[k]) {
+            if constexpr (kDefer) want[k] = app.post_d(s.pay[own[k]], w[k], tk[k], out[k], pd);
+            else want[k] = app.post(s.pay[own[k]], w[k], tk[k], out[k]);
+          }
         }
         pusher.push_n<KU>(q, want, out, P.watchdog_ns);
+      }
+      if constexpr (kDefer) {
+        // the last iteration's pending CAS (every lane of the warp reaches here together)
+        uint32_t po = 0;
+        const bool pw = app.resolve(pd, po);
+        pusher.push(q, pw, po, P.watchdog_ns);
       }
       }  // !PF
     } else if (MODE == MODE_WARP) {
