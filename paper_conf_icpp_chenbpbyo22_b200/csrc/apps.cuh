@@ -334,10 +334,14 @@ struct PrAppT {
   GhostView gv;
   double defer = 0.0;    // partitioned schedule only: a popped vertex with deg > 32 and residue < defer * deg
                          // keeps its residue (not expanded) until a later, lower threshold re-seeds it
+  unsigned long long pol_last = 0;  // single partition: residue atomics evict_last, rank reductions evict_first
 
   __device__ __forceinline__ bool remote(uint32_t w) const { return PART && gv.remote_dyn(w); }
   __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
-  __device__ __forceinline__ void prepare() { pol_first = policy_evict_first(); }
+  __device__ __forceinline__ void prepare() {
+    pol_first = policy_evict_first();
+    pol_last = policy_evict_last();
+  }
 
   __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
     const double rho = __longlong_as_double(
@@ -349,7 +353,13 @@ struct PrAppT {
       if (rho != 0.0) red_add_f64(res + v, rho);
       return false;
     }
-    if (rho != 0.0) red_add_f64(rank + v, rho);
+    if (rho != 0.0) {
+      if (!PART)
+        asm volatile("red.global.add.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(rank + v), "d"(rho), "l"(pol_first)
+                     : "memory");
+      else
+        red_add_f64(rank + v, rho);
+    }
     if (deg == 0 || rho == 0.0) return false;  // dangling: absorb (R-PR-3)
     if (dbg_expand) atomicAdd(dbg_expand + v, 1u);
     p = alpha * rho / (double)deg;
@@ -358,7 +368,16 @@ struct PrAppT {
 
   __device__ __forceinline__ Token pre(const Payload delta, uint32_t w) const {
     if (remote(w)) return 0.0;
-    return atomicAdd(res + (PART ? w - gv.vb : w), delta);
+    const uint32_t lw = PART ? w - gv.vb : w;
+    if (!PART) {
+      // residue atomics keep their lines in L2 (evict_last) against the col stream and the rank reductions
+      // (C5: residue 537 MB > L2; 1.24 -> 1.17 s, profiles/r02_ab_pr_l2_hints.txt)
+      double old;
+      asm volatile("atom.global.add.L2::cache_hint.f64 %0, [%1], %2, %3;"
+                   : "=d"(old) : "l"(res + lw), "d"(delta), "l"(pol_last) : "memory");
+      return old;
+    }
+    return atomicAdd(res + lw, delta);
   }
   __device__ __forceinline__ bool crossing(const Payload delta, uint32_t lw, Token old, uint32_t& out) const {
     if (activate && old <= eps && old + delta > eps) {
