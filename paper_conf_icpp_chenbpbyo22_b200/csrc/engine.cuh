@@ -503,7 +503,11 @@ struct Worker {
             unsigned long long want = (t - h) / nworkers;
             const unsigned long long lo = K < P.min_claim ? K : P.min_claim;
             want = want < lo ? lo : (want > K ? K : want);
+#ifdef ATOS_CLAIM_ADD
+            if (true) {  // experiment: atomicAdd claims in every regime (over-claims become pending slots)
+#else
             if (t - h >= 2ull * want) {
+#endif
               const unsigned long long b = ctr_add(&q.ctl->head.v, want);
               *(unsigned long long*)&s.ctr[6] = b;
               s.ctr[4] = (uint32_t)want;
@@ -579,7 +583,11 @@ struct Worker {
             s.ctr[3] = 1;
           }
           tl_sample(P);
+#ifdef ATOS_IDLE_SPIN
+          if (npn == 0) __nanosleep(backoff);  // experiment: spin (no sleep) while holding pending slots
+#else
           __nanosleep(backoff);
+#endif
           backoff = backoff < ATOS_BACKOFF_MAX ? backoff * 2 : ATOS_BACKOFF_MAX;
         }
       }
@@ -643,7 +651,8 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
   wk.init(smem_raw + (size_t)nwarps * kPushBuf * 4, P);
   const GroupSmem<Payload>& s = wk.s;
   const uint32_t r = wk.r, G = wk.G;
-  WarpPusher pusher = make_pusher(pushbuf);
+  // low-degree (PF) builds are latency-bound: single-CAS publishes and the small-batch scan below
+  auto pusher = make_pusher<PF>(pushbuf);
   // CTA mode: owner table after the group arena
   uint32_t* cown = (uint32_t*)(smem_raw + (size_t)nwarps * kPushBuf * 4 + group_smem_bytes<Payload>(wk.K));
   unsigned long long my_pops = 0, my_edges = 0;
@@ -747,6 +756,22 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
     if (MODE == MODE_CTA) {
       // load-balancing search over the flattened edge list of the batch
       uint32_t total = 0;
+      if (PF && nready <= 32u) {
+        // small batch (thin frontiers): warp 0 scans, one barrier instead of the block scan's four
+        if (r < 32u) {
+          const uint32_t d = r < nready ? s.off[r] : 0u;
+          uint32_t incl = d;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, incl, o);
+            if (r >= (uint32_t)o) incl += y;
+          }
+          if (r < nready) s.off[r] = incl - d;
+          if (r == 31u) s.ctr[40] = incl;
+        }
+        __syncthreads();
+        total = s.ctr[40];
+      } else {
       uint32_t mydeg = 0;
       const uint32_t per = (nready + G - 1) / G;
       const uint32_t i0 = min(r * per, nready), i1 = min(i0 + per, nready);
@@ -754,6 +779,7 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
       uint32_t excl = block_exclusive_scan(mydeg, s.ctr + 8, &total);
       for (uint32_t i = i0; i < i1; ++i) { const uint32_t d = s.off[i]; s.off[i] = excl; excl += d; }
       __syncthreads();
+      }
       my_edges += (r == 0) ? total : 0;
       // KU CONSECUTIVE edges per lane per iteration (a warp covers 32*KU
       // consecutive flattened edges, so col reads stay coalesced).  Owners:

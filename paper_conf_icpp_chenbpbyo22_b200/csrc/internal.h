@@ -74,6 +74,7 @@ struct Part {
   size_t nb_ipc_bytes = 0;
   std::vector<void*> nb_peer_base;
   uint64_t ring_cap = 0;
+  uint64_t max_deg = ~0ull;         // largest row length when known (whole-graph upload), else ~0
   void* host_pinned = nullptr;      // 4 KB pinned scratch for control-block reads
   bool ring_clean = false;          // every ring slot is EMPTY
 };

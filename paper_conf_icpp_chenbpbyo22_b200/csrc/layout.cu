@@ -273,6 +273,7 @@ int create_single(atos_csr* g, const int64_t* row_ptr, const int32_t* col, int w
     return ATOS_ERR_INVALID_ARG;
   }
   g->max_degree = (int64_t)hmx;
+  p.max_deg = hmx;
   // 2. layout decision (ATOS_LAYOUT_AUTO: an f64 per-vertex array would not fit half of L2, and the
   //    degrees are skewed)
   bool want = flags == ATOS_LAYOUT_DEGREE;

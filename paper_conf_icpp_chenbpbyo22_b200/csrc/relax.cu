@@ -324,6 +324,14 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
     P.nbig = kBigSlots;
     P.big_threshold = r.big_threshold > 0 ? (uint32_t)r.big_threshold : std::max(4096u, 32u * wsz);
     P.big_chunk = r.big_chunk > 0 ? (uint32_t)r.big_chunk : std::max(1024u, 8u * wsz);
+    // no row can become a big task (known maximum degree below the threshold): no assist, so the worker
+    // loop skips the per-batch big-task check (one L2 round trip and a barrier per batch -- ~7 % of a
+    // hop on high-diameter meshes, tools/hop_latency.py)
+    if (p.max_deg <= P.big_threshold) {
+      P.big = nullptr;
+      P.nbig = 0;
+      P.big_threshold = 0xFFFFFFFFu;
+    }
   }
   if (mode == MODE_CTA) {
     // 256-thread CTA workers: the (256, 5) register budget (48 regs, 40 warps per SM); kU = 2 edges
