@@ -68,6 +68,12 @@ struct BfsAppT {
   // fused consume + begin (engine.cuh consume_slot_fused): begin() only clears the queued flag / reads the
   // depth, so a speculative begin on a slot lost to a lapping producer can at worst cause a duplicate push
   static constexpr bool kFusedBegin = ATOS_FUSED_BEGIN != 0 && !PART;
+  // CAS first (the low-degree PF builds, engine.cuh): no prefilter load -- the CAS guesses "unvisited" and
+  // a visited target fails it, returning the word the prefilter would have read.  On a high-diameter graph
+  // the prefilter costs one round trip per hop, two past depth 254 (the u8 shadow saturates there and the
+  // depth word is read as well).
+  static constexpr bool kCasFirst = !PART;
+  static constexpr uint32_t kBlind = 0xFFFFFFFFu;  // the token that means "no prefilter read"
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
   const uint32_t* __restrict__ row_ptr;
@@ -111,7 +117,7 @@ struct BfsAppT {
   // relax local vertex lw with candidate depth nd; true -> enqueue lw
   __device__ __forceinline__ bool relax_local(const Payload nd, uint32_t lw, Token tok, uint32_t& out) const {
     uint32_t expect = 0xFFFFFFFFu;  // guess: unvisited
-    if (shadow) {
+    if (shadow && tok != kBlind) {
       if (tok != 255u && tok <= nd) return false;
       if (nd >= 255u) {  // shadow carries no information at this depth: prefilter on the word
         asm volatile("ld.global.u32 %0, [%1];" : "=r"(expect) : "l"(depth + lw));

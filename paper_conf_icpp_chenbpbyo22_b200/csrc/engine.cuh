@@ -323,6 +323,12 @@ struct PendOf<A, true> {
   using type = typename A::Pend;
 };
 
+// apps whose relax can start with the CAS instead of a prefilter read (BfsAppT::kCasFirst, token kBlind)
+template <class A, class = void>
+struct has_cas_first : std::false_type {};
+template <class A>
+struct has_cas_first<A, std::void_t<decltype(A::kCasFirst)>> : std::bool_constant<A::kCasFirst> {};
+
 // Per-group shared-memory arena.  K = items a group may hold at once.
 template <class Payload>
 struct GroupSmem {
@@ -608,6 +614,9 @@ struct Worker {
 
   // All pushes of the batch are published (every warp flushed before this):
   // count the batch as done with release semantics.
+  // LEAN (the latency-bound PF builds): no trailing barrier -- the batch's shared state is dead after the
+  // first one, and the next claim's barrier waits for the leader anyway
+  template <bool LEAN = false>
   __device__ __forceinline__ void complete(const EngineParams& P, uint32_t nready) {
     group_sync<MODE>();
     if (PERSIST && r == 0 && nready) {
@@ -616,7 +625,7 @@ struct Worker {
       ctr_red_release(&P.q.ctl->done.v, (unsigned long long)nready);
     }
     if (r == 0) tl_sample(P);
-    group_sync<MODE>();
+    if (!LEAN) group_sync<MODE>();
   }
 };
 
@@ -729,6 +738,9 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
     if (nready == kGoBig) continue;
     if (nready == 0) break;
     // ---------------------------------------------------------- begin (per item)
+    // (PF builds, fused pops, no assist: the pass below would only copy the gather's results in place)
+    const bool skip_begin = PF && kFused && !assist;
+    if (!skip_begin) {
     for (uint32_t k = r; k < nready; k += G) {
       uint32_t st = 0, dg = 0;
       Payload p{};
@@ -748,6 +760,7 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
       s.pay[k] = p;
     }
     group_sync<MODE>();
+    }
     ATOS_PH(PH_BEGIN);
     my_pops += (r == 0) ? nready : 0;
     const uint32_t deferred = s.ctr[5];
@@ -791,7 +804,8 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
       // owner of every wspan-edge chunk start, once per batch (a warp's span is
       // one chunk, so its owner range comes from two table reads)
       const uint32_t nchunk = (total + wspan - 1) / wspan;
-      const bool table = nchunk <= kCown;
+      // (PF builds: a batch of at most 8 chunks skips the table and its barrier; lanes 0/1 search instead)
+      const bool table = nchunk <= kCown && (!PF || nchunk > 8u);
       if (table) {
         for (uint32_t c = r; c < nchunk; c += G) {
           const uint32_t e = c * wspan;
@@ -883,7 +897,10 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
           }
 #pragma unroll
           for (int k = 0; k < KU; ++k)
-            if (own[k] != 0xFFFFu) tk[k] = app.pre(s.pay[own[k]], w[k]);
+            if (own[k] != 0xFFFFu) {
+              if constexpr (has_cas_first<App>::value) tk[k] = App::kBlind;
+              else tk[k] = app.pre(s.pay[own[k]], w[k]);
+            }
 #pragma unroll
           for (int k = 0; k < KU; ++k) {
             want[k] = false;
@@ -1088,7 +1105,7 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
       ph_acc[lo ? PH_EDGES_LO : PH_EDGES_HI] += ph_total;
     }
 #endif
-    wk.complete(P, nready - deferred);
+    wk.template complete<PF>(P, nready - deferred);
     ATOS_PH(PH_COMPLETE);
   }
   ATOS_PH_FLUSH();
