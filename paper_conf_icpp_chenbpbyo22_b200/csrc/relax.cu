@@ -303,7 +303,10 @@ static int launch_relax_inner(const App& app, const Ring& q, const Resolved& r, 
   P.fetch = (uint32_t)r.fetch;
   P.watchdog_ns = r.watchdog_ns;
   P.h0 = P.t0 = 0;
-  P.min_claim = min_claim_for(kMinClaim);
+  // smallest fair-share claim: 24 items on low-degree graphs (m < 8n: meshes / road-like, whose thin
+  // frontiers are chains of small batches -- C2 mesh 30.1 -> 28.7 ms, road-like 42.4 -> 40.4 ms vs 16,
+  // profiles/r02_ab_min_claim.txt), 16 otherwise
+  P.min_claim = min_claim_for(p.n_local > 0 && p.m_local < 8 * p.n_local ? 24u : (uint32_t)kMinClaim);
   const int mode = mode_of(r.worker);
   const int block = mode == MODE_CTA ? r.worker : r.block_threads;
   // hub assist (persistent CTA / warp workers): auto threshold = 32 edges per
