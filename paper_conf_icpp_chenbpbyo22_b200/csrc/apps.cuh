@@ -72,7 +72,10 @@ struct BfsAppT {
   // a visited target fails it, returning the word the prefilter would have read.  On a high-diameter graph
   // the prefilter costs one round trip per hop, two past depth 254 (the u8 shadow saturates there and the
   // depth word is read as well).
-  static constexpr bool kCasFirst = !PART;
+#ifndef ATOS_CAS_FIRST
+#define ATOS_CAS_FIRST 1
+#endif
+  static constexpr bool kCasFirst = ATOS_CAS_FIRST != 0 && !PART;
   static constexpr uint32_t kBlind = 0xFFFFFFFFu;  // the token that means "no prefilter read"
   using Payload = uint32_t;  // d + 1
   using Token = uint32_t;    // prefilter value (shadow byte, or depth word)
