@@ -212,6 +212,21 @@ def test_byte_state_depth_boundary(n, deep):
         assert st2["flags"] == 0
 
 
+@pytest.mark.parametrize("src", [0, 1733, 2999])
+def test_deep_path_thin_chain(src):
+    """The thin-frontier chain of the low-degree builds (CAS-first u32 relax, warp-0 scan, single-CAS
+    publish, lean completion, no assist without big rows) on a 3000-vertex path: one vertex per level, depths
+    far past the u8 shadow's 254 -- closed form |i - src| for every worker / grid / dedupe / discrete mode."""
+    n = 3000
+    rp, ci = G.path(n)
+    csr = csr_of(rp, ci)
+    want = np.abs(np.arange(n) - src).astype(np.uint32)
+    for knobs in (dict(), dict(num_blocks=1), dict(num_blocks=3), dict(dedupe=0), dict(worker=32, fetch_size=4),
+                  dict(persistent=0), dict(depth_state=2), dict(worker=1024, fetch_size=1024)):
+        d, _ = atos.bfs(csr, src, **knobs)
+        np.testing.assert_array_equal(as_u32(d), want, err_msg=str(knobs))
+
+
 def test_byte_state_word_neighbours():
     """Four consecutive vertex ids share one 32-bit state word: a 4-clique plus pendant chains
     exercises CAS retries on neighbouring bytes."""
