@@ -98,7 +98,7 @@ typedef struct {
     int      worker;            /* 1 thread, 32 warp, 64..1024 CTA; 0 = per-app default (CTA: BFS 256, PageRank 512,
                                    colouring 1024) */
     int      fetch_size;        /* items per pop per worker (FETCH_SIZE); 0 = default (CTA: worker size
-                                   for BFS, min(worker,256) for PageRank, min(worker,128) for colouring; warp 8;
+                                   for BFS, min(worker,256) for PageRank, min(worker,48) for colouring; warp 8;
                                    thread 1) */
     int      num_blocks;        /* 0 = occupancy max (persistent) / proportional to the frontier (discrete) */
     int      block_threads;     /* threads per block for thread/warp workers; 0 = 256 */
