@@ -322,6 +322,15 @@ struct BfsByteAppT {
 // Activation (DESIGN.md R-PR-6): w is pushed iff its residue crosses eps from
 // below (old <= eps < old + delta, evaluated in the same fp64 rounding as the
 // atomic), which keeps "residue[v] > eps  =>  v queued or in flight".
+// Residue slot of vertex v (single-partition PageRank on a degree-layout graph, rs_log = log2 T > 0): the
+// 16T highest-degree vertices are spread as (v mod T) * 16 + v / T so that each of the T hottest owns a whole
+// 128-byte line of the f64 residue array -- same-line atomics serialise in the L2 atomic unit -- while the ids
+// themselves stay packed by degree (what the BFS byte state wants).  A bijection on [0, n) (16T <= n).
+__host__ __device__ __forceinline__ uint32_t res_slot(uint32_t v, uint32_t rs_log) {
+  if (rs_log == 0 || v >= (16u << rs_log)) return v;
+  return ((v & ((1u << rs_log) - 1u)) << 4) | (v >> rs_log);
+}
+
 template <bool PART>
 struct PrAppT {
   static constexpr bool kAcquirePop = true;  // atomicExch must follow the pusher's crossing add
@@ -344,6 +353,7 @@ struct PrAppT {
   double defer = 0.0;    // partitioned schedule only: a popped vertex with deg > 32 and residue < defer * deg
                          // keeps its residue (not expanded) until a later, lower threshold re-seeds it
   unsigned long long pol_last = 0;  // single partition: residue atomics evict_last, rank reductions evict_first
+  uint32_t rs_log = 0;              // single partition on a degree-layout graph: residue and rank slots (res_slot)
 
   __device__ __forceinline__ bool remote(uint32_t w) const { return PART && gv.remote_dyn(w); }
   __device__ __forceinline__ uint32_t neighbor(uint32_t e) const { return ld_stream(col + e, pol_first); }
@@ -354,7 +364,7 @@ struct PrAppT {
 
   __device__ __forceinline__ bool begin(uint32_t v, uint32_t& start, uint32_t& deg, Payload& p) const {
     const double rho = __longlong_as_double(
-        (long long)atomicExch((unsigned long long*)(res + v), 0ull));
+        (long long)atomicExch((unsigned long long*)(res + (PART ? v : res_slot(v, rs_log))), 0ull));
     start = __ldg(row_ptr + v);
     deg = __ldg(row_ptr + v + 1) - start;
     if (PART && defer > 0.0 && deg > 32 && rho < defer * (double)deg) {
@@ -364,7 +374,8 @@ struct PrAppT {
     }
     if (rho != 0.0) {
       if (!PART)
-        asm volatile("red.global.add.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(rank + v), "d"(rho), "l"(pol_first)
+        asm volatile("red.global.add.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(rank + res_slot(v, rs_log)), "d"(rho),
+                     "l"(pol_first)
                      : "memory");
       else
         red_add_f64(rank + v, rho);
@@ -383,7 +394,7 @@ struct PrAppT {
       // (C5: residue 537 MB > L2; 1.24 -> 1.17 s, profiles/r02_ab_pr_l2_hints.txt)
       double old;
       asm volatile("atom.global.add.L2::cache_hint.f64 %0, [%1], %2, %3;"
-                   : "=d"(old) : "l"(res + lw), "d"(delta), "l"(pol_last) : "memory");
+                   : "=d"(old) : "l"(res + res_slot(lw, rs_log)), "d"(delta), "l"(pol_last) : "memory");
       return old;
     }
     return atomicAdd(res + lw, delta);

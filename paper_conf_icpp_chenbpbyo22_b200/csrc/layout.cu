@@ -7,8 +7,9 @@
 // PageRank residue is 537 MB, L2 126 MB) most of the per-edge f64 atomics miss
 // L2.  At creation the CSR is relabelled once:
 //   rank r = position of v in descending-degree order (stable, by old id);
-//   new id = r, except that the first 16*T ranks are interleaved as
-//            (r mod T) * 16 + r / T  (T = min(4096, n / 16)),
+//   new id = r (T = 1 since round 2: the interleave below moved into PageRank's residue addressing,
+//            apps.cuh res_slot); with T > 1 (ATOS_LAYOUT_T) the first 16*T ranks are interleaved as
+//            (r mod T) * 16 + r / T,
 // which packs the hot set into a prefix of the state arrays (L2-resident) but
 // gives each of the T hottest vertices its own 128-byte line of an f64 array,
 // so the hubs' atomics do not serialise on shared lines/slices (without the
@@ -17,7 +18,8 @@
 // 14.7 -> 13.2 ms, C3 within 3 %.  The interleave width T trades the two C5 workloads (tools/layout_probe.py,
 // profiles/r02_layout_interleave.txt): the BFS byte state wants the hubs packed (32 per sector), the PageRank
 // f64 residues want them apart -- T = 65536 / 4096 / 1 (none): BFS 13.15 / 12.77 / 12.59 ms, PageRank 1173 /
-// 1192 / 1775 ms; T = 4096 (the top 64 K ranks interleaved) keeps PageRank within 2 % and BFS -3 %.
+// 1192 / 1775 ms.  Since round 2 the ids use T = 1 and PageRank interleaves its own residue / rank arrays
+// (apps.cuh res_slot): BFS 12.6 ms and PageRank 1.19 s at once.
 //
 // The method is unchanged: every call maps the source into the internal ids
 // and scatters its output back (out[old] = result[new]); colouring seeds its
@@ -133,7 +135,9 @@ __global__ void __launch_bounds__(kRemapThreads) k_layout_remap(const uint32_t* 
 // o2n / n2o and the new offsets rp_new[n+1] from the (narrowed) old offsets; `base` = per-old-row shift.
 int layout_prepare(atos_csr* g, const uint32_t* rp_old, int64_t n, int64_t m, cudaStream_t s, DevBuf& rp_new,
                    DevBuf& base) {
-  uint32_t T = (uint32_t)std::min<int64_t>(4096, n / 16);
+  // T = 1: no interleave of the ids (the BFS byte state wants the hubs packed); single-partition PageRank
+  // spreads its residues itself (res_slot in apps.cuh)
+  uint32_t T = 1;
   if (const char* e = getenv("ATOS_LAYOUT_T")) T = (uint32_t)std::max<int64_t>(1, std::min<int64_t>(atol(e), n / 16));
   struct Scratch {  // released on every return path
     DevBuf deg, ids, deg_s, order, ndeg, tmp;

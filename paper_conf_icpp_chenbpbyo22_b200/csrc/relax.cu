@@ -116,7 +116,7 @@ __device__ __forceinline__ uint32_t row_of(const uint32_t* __restrict__ row_ptr,
 // bound the tile's rows, then each thread searches only that (L1-resident)
 // row range -- load-balanced regardless of hub degrees.
 __global__ void k_pr_init_edges(const uint32_t* __restrict__ row_ptr, const uint32_t* __restrict__ col,
-                                double* res, uint32_t n, uint32_t m, double c) {
+                                double* res, uint32_t n, uint32_t m, double c, uint32_t rs_log = 0) {
   __shared__ uint32_t s_r[2];
   for (uint64_t t0 = (uint64_t)blockIdx.x * blockDim.x; t0 < m; t0 += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t e0 = (uint32_t)t0;
@@ -129,24 +129,37 @@ __global__ void k_pr_init_edges(const uint32_t* __restrict__ row_ptr, const uint
     if (e <= e1) {
       const uint32_t v = row_of(row_ptr, s_r[0], s_r[1], e);
       const uint32_t deg = __ldg(row_ptr + v + 1) - __ldg(row_ptr + v);
-      red_add_f64(res + __ldg(col + e), c / (double)deg);
+      red_add_f64(res + res_slot(__ldg(col + e), rs_log), c / (double)deg);
     }
     __syncthreads();
   }
 }
 
 // Initial frontier (R-PR-7): every vertex with residue > eps, warp-aggregated pushes.
-__global__ void k_pr_seed(const double* res, int64_t n, double eps, Ring q, unsigned long long wd) {
+__global__ void k_pr_seed(const double* res, int64_t n, double eps, Ring q, unsigned long long wd,
+                          uint32_t rs_log = 0) {
   __shared__ uint32_t bufs[32 * kPushBuf];
   WarpPusher pusher = make_pusher(bufs);
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n; base += stride) {
     const int64_t v = base + threadIdx.x;
-    const bool want = v < n && res[v] > eps;
+    const bool want = v < n && res[res_slot((uint32_t)v, rs_log)] > eps;
     pusher.push(q, want, (uint32_t)v, wd);
   }
   pusher.flush(q, wd);
   if (lane_id() == 0) atomicAdd(&q.ctl->stat_pushes.v, (unsigned long long)pusher.total);
+}
+
+// Slot-addressed accumulation (res_slot, rs_log > 0): rank_out[v] = acc[slot(v)] / n, residual sum as below.
+__global__ void k_pr_finalize_slots(const double* acc, double* rank, const double* res, int64_t n, double n_global,
+                                    uint32_t rs_log, double* sum) {
+  double a = 0.0;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+    rank[v] = acc[res_slot((uint32_t)v, rs_log)] / n_global;
+    a += res[v];
+  }
+  for (int o = 16; o; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+  if (lane_id() == 0 && a != 0.0) atomicAdd(sum, a);
 }
 
 // rank_out = rank / n_global (R-PR-4); residual sum into *sum (conservation check).
@@ -165,7 +178,7 @@ __global__ void k_pr_finalize_n(double* rank, const double* res, int64_t n, doub
 // Check_Size ids with one atomicAdd on the check cursor and enqueue those with
 // residue > eps.  (The sweep variant drives activation; see pagerank_single.)
 __global__ void k_pr_sweep(const double* res, int64_t n, double eps, Ring q, uint32_t check_size,
-                           unsigned long long wd) {
+                           unsigned long long wd, uint32_t rs_log = 0) {
   __shared__ uint32_t bufs[32 * kPushBuf];
   __shared__ unsigned long long s_c;
   WarpPusher pusher = make_pusher(bufs);
@@ -178,7 +191,8 @@ __global__ void k_pr_sweep(const double* res, int64_t n, double eps, Ring q, uin
     if (c >= (unsigned long long)n) break;
     for (uint32_t i = 0; i < check_size; i += blockDim.x) {
       const unsigned long long id = c + i + threadIdx.x;
-      const bool want = (i + threadIdx.x) < check_size && id < (unsigned long long)n && res[id] > eps;
+      const bool want = (i + threadIdx.x) < check_size && id < (unsigned long long)n &&
+                        res[res_slot((uint32_t)id, rs_log)] > eps;
       pusher.push(q, want, (uint32_t)id, wd);
     }
   }
@@ -489,20 +503,32 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
   Ring q = ring_of(p);
   k_run_begin<<<1, 32, 0, s>>>(q.ctl);
   g_launches++;
+  // residue slots on a degree-layout graph: T = 65536 (or the largest power of two with 16T <= n)
+  uint32_t rs_log = 0;
+  if (g->relabeled && g->parts.size() == 1)
+    while (rs_log < 16 && (16ll << (rs_log + 1)) <= n) ++rs_log;
+  if (const char* e = getenv("ATOS_PR_SLOT_LOG")) rs_log = (uint32_t)std::max(0, std::min(atoi(e), (int)rs_log));
   const int gs = 148 * 8;
+  // slot-addressed rank accumulator (the caller's buffer receives rank_out in vertex order at the end)
+  double* const rank_out = rank;
+  if (rs_log) {
+    ATOS_TRY(p.vbuf_b.ensure((size_t)n * 8));
+    rank = p.vbuf_b.as<double>();
+  }
   k_pr_init_vertices<<<gs, 256, 0, s>>>(rank, res, n, 1.0 - alpha);
   g_launches++;
   if (p.m_local > 0) {
     k_pr_init_edges<<<gs * 2, 256, 0, s>>>(p.row_ptr, p.col, res, (uint32_t)n, (uint32_t)p.m_local,
-                                            (1.0 - alpha) * alpha);
+                                            (1.0 - alpha) * alpha, rs_log);
     g_launches++;
   }
-  k_pr_seed<<<gs, 1024, 0, s>>>(res, n, eps, q, r.watchdog_ns);
+  k_pr_seed<<<gs, 1024, 0, s>>>(res, n, eps, q, r.watchdog_ns, rs_log);
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   if (r.l2_persist) set_l2_window(s, res, (size_t)n * 8, true);
   PrApp app{p.row_ptr, p.col, 0ull, rank, res, alpha, eps, r.check_size > 0 ? 0 : 1, nullptr,
             GhostView{0u, (uint32_t)n, nullptr, nullptr, nullptr}};
+  app.rs_log = rs_log;
   uint32_t* dbg_edge = nullptr;
   const bool dbg = getenv("ATOS_DEBUG_EDGES") != nullptr;
   if (dbg) {
@@ -534,7 +560,7 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
       if (h[1] != 0) break;  // watchdog/overflow: reported by finish_queue
       const unsigned long long t_before = h[0];
       ATOS_CUDA(cudaMemsetAsync(&q.ctl->check.v, 0, 8, s));
-      k_pr_sweep<<<gs, 256, 0, s>>>(res, n, eps, q, (uint32_t)r.check_size, r.watchdog_ns);
+      k_pr_sweep<<<gs, 256, 0, s>>>(res, n, eps, q, (uint32_t)r.check_size, r.watchdog_ns, rs_log);
       g_launches++;
       ATOS_CUDA(cudaMemcpyAsync(h, &q.ctl->tail.v, 8, cudaMemcpyDeviceToHost, s));
       ATOS_TRY(stream_wait(s, r.timeout_s));
@@ -570,7 +596,8 @@ int pagerank_single(atos_csr* g, Part& p, double alpha, double eps, double* rank
   }
   if (rc != ATOS_OK) return rc;
   ATOS_CUDA(cudaMemsetAsync(sum, 0, 8, s));
-  k_pr_finalize_n<<<gs, 256, 0, s>>>(rank, res, n, (double)n, sum);
+  if (rs_log) k_pr_finalize_slots<<<gs, 256, 0, s>>>(rank, rank_out, res, n, (double)n, rs_log, sum);
+  else k_pr_finalize_n<<<gs, 256, 0, s>>>(rank, res, n, (double)n, sum);
   g_launches++;
   ATOS_CUDA(cudaGetLastError());
   rc = finish_queue(p, s, st, "pagerank");
