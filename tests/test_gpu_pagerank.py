@@ -117,3 +117,40 @@ def test_layout_input_and_auto_agree(rmat13):
         csr = atos.CSR.from_graph(g.to(DEV), layout=layout)
         r, st = atos.pagerank(csr, 0.85, 1e-6)
         check_pr(rp, ci, r, st, 1e-6, ref=ref)
+
+
+@pytest.fixture(scope="module")
+def rmat13_degree(rmat13):
+    rp, ci, ref, _ = rmat13
+    g = gen.Graph(len(rp) - 1, len(ci), torch.from_numpy(rp), torch.from_numpy(ci))
+    return rp, ci, ref, atos.CSR.from_graph(g.to(DEV), layout="degree")
+
+
+@pytest.mark.parametrize("knobs", KNOBS, ids=kid)
+def test_degree_layout_residue_slots(rmat13_degree, knobs):
+    """Single-partition PageRank on a degree-layout graph keeps its residue and rank arrays in interleaved
+    slots (apps.cuh res_slot): init, seed, relax, the Check_Size sweep and the finalize all go through the
+    same bijection -- every worker mode stays in the north-star tolerance with conservation."""
+    rp, ci, ref, csr = rmat13_degree
+    r, st = atos.pagerank(csr, 0.85, 1e-6, **knobs)
+    err = check_pr(rp, ci, r, st, 1e-6, ref=ref)
+    assert abs(err) < 1e-9 * len(ref)
+
+
+@pytest.mark.parametrize("slot_log", ["0", "1", "4"])
+def test_degree_layout_slot_widths(rmat13_degree, slot_log, monkeypatch):
+    """Other interleave widths (ATOS_PR_SLOT_LOG; 0 = plain addressing) give the same fixed point."""
+    monkeypatch.setenv("ATOS_PR_SLOT_LOG", slot_log)
+    rp, ci, ref, csr = rmat13_degree
+    r, st = atos.pagerank(csr, 0.85, 1e-6)
+    check_pr(rp, ci, r, st, 1e-6, ref=ref)
+
+
+def test_degree_layout_tiny_graphs():
+    """n below 32 (no room for an interleave) and a star (one hub) under the degree layout."""
+    for rp, ci in (G.path(7), G.star(40), G.complete(12)):
+        n = len(rp) - 1
+        g = gen.Graph(n, len(ci), torch.from_numpy(rp), torch.from_numpy(ci))
+        csr = atos.CSR.from_graph(g.to(DEV), layout="degree")
+        r, st = atos.pagerank(csr, 0.85, 1e-8)
+        check_pr(rp, ci, r, st, 1e-8)
