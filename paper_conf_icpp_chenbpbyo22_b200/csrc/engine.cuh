@@ -509,11 +509,7 @@ struct Worker {
             unsigned long long want = (t - h) / nworkers;
             const unsigned long long lo = K < P.min_claim ? K : P.min_claim;
             want = want < lo ? lo : (want > K ? K : want);
-#ifdef ATOS_CLAIM_ADD
-            if (true) {  // experiment: atomicAdd claims in every regime (over-claims become pending slots)
-#else
             if (t - h >= 2ull * want) {
-#endif
               const unsigned long long b = ctr_add(&q.ctl->head.v, want);
               *(unsigned long long*)&s.ctr[6] = b;
               s.ctr[4] = (uint32_t)want;
@@ -589,11 +585,7 @@ struct Worker {
             s.ctr[3] = 1;
           }
           tl_sample(P);
-#ifdef ATOS_IDLE_SPIN
-          if (npn == 0) __nanosleep(backoff);  // experiment: spin (no sleep) while holding pending slots
-#else
           __nanosleep(backoff);
-#endif
           backoff = backoff < ATOS_BACKOFF_MAX ? backoff * 2 : ATOS_BACKOFF_MAX;
         }
       }
