@@ -174,9 +174,9 @@ ATOS_API int atos_csr_create(atos_csr** out, int64_t n, int64_t m, const int64_t
 /*
  * atos_csr_create with layout flags.  atos_csr_create(...) == atos_csr_create_ex(..., 0).
  *   ATOS_LAYOUT_DEGREE: a single-partition graph is stored in the DEGREE LAYOUT -- vertices relabelled
- *     once, at creation, by descending degree with the 65536 hottest interleaved one per 128-byte line
- *     of an f64 state array -- so the hubs' per-vertex state is a compact
- *     L2-resident prefix.  Invisible to the caller: sources are mapped in, outputs are written in the
+ *     once, at creation, by descending degree -- so the hubs' per-vertex state is
+ *     a compact L2-resident prefix (single-partition PageRank additionally spreads its residue / rank
+ *     arrays so that each of the 65536 hottest vertices owns a 128-byte line).  Invisible to the caller: sources are mapped in, outputs are written in the
  *     caller's vertex ids, colouring seeds its queue in the caller's id order.  Costs two u32[n] maps
  *     on the device and one output scatter per call.
  *   ATOS_LAYOUT_AUTO (0): the degree layout when it pays -- an f64 per-vertex array would not fit half
