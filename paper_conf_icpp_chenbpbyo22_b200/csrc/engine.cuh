@@ -985,6 +985,36 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
         }
 #else
         const uint32_t e0 = wfirst + lane_id() * KU;
+#ifndef ATOS_OWN_FILL
+#define ATOS_OWN_FILL 1
+#endif
+        if (ATOS_OWN_FILL && KU * 32u <= 128u && nchunk + 32u * nwarps <= kCown && ohi - olo >= 8u &&
+            ohi - olo < 255u) {
+          // a span over many short rows (warp-uniform): instead of a binary search plus a walk per lane, the
+          // lanes write each row's owner offset over its edges into a per-warp byte map (the owner table's
+          // unused tail: 128 B = 32 words per warp) -- rows are disjoint, so every byte has one writer -- and every lane
+          // reads its KU owners back with one shared-memory load each
+          uint8_t* own_s = (uint8_t*)(cown + kCown - 32u * nwarps) + warp_id() * 128u;
+          __syncwarp();  // the previous span's reads are done
+          for (uint32_t it = olo + lane_id(); it <= ohi; it += 32u) {
+            const uint32_t a = max(s.off[it], wfirst);
+            const uint32_t b = min(it + 1u < nready ? s.off[it + 1u] : total, wfirst + wspan);
+            for (uint32_t e = a; e < b; ++e) own_s[e - wfirst] = (uint8_t)(it - olo);
+          }
+          __syncwarp();
+#pragma unroll
+          for (int k = 0; k < KU; ++k) {
+            const uint32_t e = e0 + k;
+            val[k] = e < total;
+            if (val[k]) {
+              const uint32_t o = olo + own_s[e - wfirst];
+              own[k] = o;
+              const uint32_t ce = s.start[o] + (e - s.off[o]);
+              w[k] = app.neighbor(ce);
+              ATOS_DBG_EDGE(P, ce);
+            }
+          }
+        } else {
         uint32_t o = olo;
         {
           uint32_t l = olo, h = ohi + 1;
@@ -1005,6 +1035,7 @@ __global__ void __launch_bounds__(MINB == 1 ? ATOS_MAXT : 256, MINB) k_relax_wor
             w[k] = app.neighbor(ce);
             ATOS_DBG_EDGE(P, ce);
           }
+        }
         }
 #endif
 #pragma unroll
